@@ -1,0 +1,138 @@
+/*
+ * cszp2.h — C ABI of the B200-native cuSZp2 compressor (libcszp2.so).
+ *
+ * Implements the single-kernel error-bounded lossy compressor of
+ *   Huang, Di, Li, Cappello, "cuSZp2: A GPU Lossy Compressor with Extreme
+ *   Throughput and Optimized Compression Ratio", SC'24 (PAPER.md; P:n = line n)
+ * for f32 / f64 fields on sm_100a. The stream format and the arithmetic
+ * contract are FORMAT.md (repo root).
+ *
+ * Conventions for every entry point:
+ *  - Plain pointers and sizes only; `stream` is a cudaStream_t passed as void*
+ *    (NULL = legacy default stream). Pointers named d_* are DEVICE pointers,
+ *    h_* are HOST pointers.
+ *  - The caller owns every buffer; the library allocates nothing and keeps no
+ *    state between calls. Calls on different streams with disjoint buffers may
+ *    run concurrently.
+ *  - Work is enqueued on `stream` without host synchronisation, except where
+ *    a function says it synchronises.
+ *  - Return value: CSZP2_OK, or a synchronous error (bad argument, CUDA launch
+ *    failure). Data-dependent failures are reported inside the stream header
+ *    (status byte) and through d_status, never by the return value.
+ *  - Alignment: d_in, d_out, d_cmp must be 16-byte aligned (TMA requirement);
+ *    cudaMalloc'd pointers are.
+ */
+#ifndef CSZP2_H
+#define CSZP2_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* status / error codes */
+#define CSZP2_OK 0
+#define CSZP2_ERR_ARG 1    /* invalid argument (null pointer, dtype, mode, eb, alignment) */
+#define CSZP2_ERR_CUDA 2   /* a CUDA call or kernel launch failed */
+#define CSZP2_ERR_RANGE 3  /* stream status: a value's |x/2eb| exceeds 2^30-1 or is not finite (FORMAT.md §6.3) */
+#define CSZP2_ERR_FORMAT 4 /* stream is not a valid FORMAT.md v1 stream for (n, dtype) */
+
+/* dtype */
+#define CSZP2_F32 0
+#define CSZP2_F64 1
+/* error-bound mode */
+#define CSZP2_EB_ABS 0 /* |x - x'| <= eb                                   */
+#define CSZP2_EB_REL 1 /* eb = lambda; |x - x'| <= lambda * (max - min)      */
+/* lossless encoding mode */
+#define CSZP2_ENC_PLAIN 0   /* Plain-FLE for every block (CUSZP2-P)                 */
+#define CSZP2_ENC_OUTLIER 1 /* per-block Outlier-FLE when strictly smaller (CUSZP2-O) */
+
+/* Decoded stream header (FORMAT.md §3). */
+typedef struct {
+    uint32_t magic;
+    uint8_t version, dtype, enc_mode, log2L, eb_mode, status;
+    uint16_t blocks_per_tile;
+    uint64_t n;
+    double eb;      /* as given by the caller (ABS bound or REL lambda) */
+    double eb_abs;  /* bound used for quantization */
+    uint64_t payload_bytes;
+    uint64_t total_bytes;
+} cszp2_header;
+
+/* Bytes a compressed stream of n values may occupy (FORMAT.md §2); d_out of
+ * cszp2_compress must hold this many bytes. Returns 0 for an invalid dtype. */
+uint64_t cszp2_compress_bound(uint64_t n, int dtype);
+
+/* Compression (P:84-102 problem statement; Fig 4 workflow ❶-❹).
+ *  d_in        : n values of `dtype`, device, 16-byte aligned, read only.
+ *  eb          : ABS bound, or REL lambda in (0,1); finite and > 0.
+ *  d_out       : device buffer of cszp2_compress_bound(n, dtype) bytes,
+ *                16-byte aligned; receives the stream (header first).
+ *  d_out_bytes : nullable DEVICE uint64; receives the stream's total bytes
+ *                (also in the header), so a multi-GPU caller can all-gather
+ *                it without a host sync.
+ * Enqueues: a memset of the header+index region, the REL min/max kernel (REL
+ * only), and the single fused compression kernel. */
+int cszp2_compress(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
+                   int enc_mode, void *d_out, uint64_t *d_out_bytes, void *stream);
+
+/* The two phases of cszp2_compress, exposed so callers (bench.py) can time
+ * the dominant kernel alone. cszp2_compress == prepare then encode, with the
+ * same arguments. prepare: zero the header+index region of d_out and, for
+ * REL, run the device min/max reduction that writes eb_abs into the header.
+ * encode: the fused kernel (❶ quantize, in-block difference, ❷ FLE, ❸
+ * decoupled-lookback scan, ❹ concatenation). */
+int cszp2_compress_prepare(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
+                           void *d_out, void *stream);
+int cszp2_compress_encode(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
+                          int enc_mode, void *d_out, uint64_t *d_out_bytes, void *stream);
+
+/* Decompression (❸ locate → ❹ → ❷ → ❶ in one kernel).
+ *  d_cmp    : a stream produced by cszp2_compress for the same (n, dtype),
+ *             device, 16-byte aligned.
+ *  d_out    : n values of `dtype`, device, 16-byte aligned.
+ *  d_status : nullable DEVICE int. If non-null it is OR-ed with a nonzero
+ *             code (CSZP2_ERR_FORMAT / CSZP2_ERR_RANGE) when the stream is
+ *             invalid or has RANGE status (d_out is then unspecified). The
+ *             caller zeroes it beforehand. */
+int cszp2_decompress(const void *d_cmp, void *d_out, uint64_t n, int dtype, int *d_status,
+                     void *stream);
+
+/* Copy the 64-byte header of a device stream to the host and decode it.
+ * Synchronises `stream`. */
+int cszp2_read_header(const void *d_cmp, cszp2_header *h_hdr, void *stream);
+
+/* End-to-end variants with HOST buffers (bench e2e). The caller provides
+ * device work buffers (d_in_work: n*w bytes; d_out_work: compress bound);
+ * host buffers should be pinned for full PCIe speed.
+ * cszp2_compress_host: H2D copy of h_in, cszp2_compress, D2H copy of the
+ *   stream into h_out (capacity h_out_cap); *h_out_bytes = stream bytes.
+ *   Synchronises `stream`.
+ * cszp2_decompress_host: H2D copy of h_cmp (cmp_bytes) into d_cmp_work,
+ *   cszp2_decompress into d_out_work, D2H of n values into h_out.
+ *   d_status as in cszp2_decompress (nullable); its value is returned if
+ *   nonzero. Synchronises `stream`. */
+int cszp2_compress_host(const void *h_in, uint64_t n, int dtype, double eb, int eb_mode,
+                        int enc_mode, void *d_in_work, void *d_out_work, void *h_out,
+                        uint64_t h_out_cap, uint64_t *h_out_bytes, void *stream);
+int cszp2_decompress_host(const void *h_cmp, uint64_t cmp_bytes, void *d_cmp_work,
+                          void *d_out_work, void *h_out, uint64_t n, int dtype, int *d_status,
+                          void *stream);
+
+/* Multi-GPU container index: exclusive prefix sum of the
+ * per-rank stream sizes gathered from every rank's d_out_bytes.
+ *  d_sizes   : nparts device uint64 (all-gathered sizes, rank order).
+ *  d_offsets : nparts + 1 device uint64; d_offsets[r] = Σ_{j<r} d_sizes[j],
+ *              d_offsets[nparts] = total container bytes. */
+int cszp2_container_index(const uint64_t *d_sizes, int nparts, uint64_t *d_offsets,
+                          void *stream);
+
+/* Library identification ("cszp2 <version> sm_100a"). */
+const char *cszp2_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CSZP2_H */

@@ -1,0 +1,189 @@
+"""B200-native cuSZp2 (Huang et al., SC'24): error-bounded lossy compression of
+f32/f64 fields in one fused sm_100a kernel per direction.
+
+This module is a thin ctypes binding over libcszp2.so (include/cszp2.h):
+argument marshalling only. Every step of the hot path runs in the CUDA
+kernels; there is no CPU fallback — importing fails loudly if the shared
+library is missing, and calls fail if the tensors are not on a CUDA device.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+from ._build import LIB as _LIB_PATH
+
+F32, F64 = 0, 1
+EB_ABS, EB_REL = 0, 1
+ENC_PLAIN, ENC_OUTLIER = 0, 1
+OK, ERR_ARG, ERR_CUDA, ERR_RANGE, ERR_FORMAT = 0, 1, 2, 3, 4
+
+_EB = {"abs": EB_ABS, "rel": EB_REL, EB_ABS: EB_ABS, EB_REL: EB_REL}
+_ENC = {"plain": ENC_PLAIN, "outlier": ENC_OUTLIER, "p": ENC_PLAIN, "o": ENC_OUTLIER,
+        ENC_PLAIN: ENC_PLAIN, ENC_OUTLIER: ENC_OUTLIER}
+_DT = {torch.float32: F32, torch.float64: F64}
+_TORCH_DT = {F32: torch.float32, F64: torch.float64}
+
+
+class CszpError(RuntimeError):
+    def __init__(self, fn: str, rc: int):
+        super().__init__(f"{fn} failed with status {rc}")
+        self.rc = rc
+
+
+class Header(ctypes.Structure):
+    _fields_ = [
+        ("magic", ctypes.c_uint32),
+        ("version", ctypes.c_uint8), ("dtype", ctypes.c_uint8), ("enc_mode", ctypes.c_uint8),
+        ("log2L", ctypes.c_uint8), ("eb_mode", ctypes.c_uint8), ("status", ctypes.c_uint8),
+        ("blocks_per_tile", ctypes.c_uint16),
+        ("n", ctypes.c_uint64), ("eb", ctypes.c_double), ("eb_abs", ctypes.c_double),
+        ("payload_bytes", ctypes.c_uint64), ("total_bytes", ctypes.c_uint64),
+    ]
+
+    def as_dict(self) -> dict:
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+def _load():
+    if not os.path.exists(_LIB_PATH):
+        raise ImportError(
+            f"{_LIB_PATH} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'`"
+        )
+    L = ctypes.CDLL(_LIB_PATH)
+    vp, u64, i32, dbl = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int, ctypes.c_double
+    L.cszp2_compress_bound.argtypes = [u64, i32]
+    L.cszp2_compress_bound.restype = u64
+    sig = [vp, u64, i32, dbl, i32, i32, vp, vp, vp]
+    L.cszp2_compress.argtypes = sig
+    L.cszp2_compress_encode.argtypes = sig
+    L.cszp2_compress_prepare.argtypes = [vp, u64, i32, dbl, i32, vp, vp]
+    L.cszp2_decompress.argtypes = [vp, vp, u64, i32, vp, vp]
+    L.cszp2_read_header.argtypes = [vp, ctypes.POINTER(Header), vp]
+    L.cszp2_compress_host.argtypes = [vp, u64, i32, dbl, i32, i32, vp, vp, vp, u64,
+                                      ctypes.POINTER(ctypes.c_uint64), vp]
+    L.cszp2_decompress_host.argtypes = [vp, u64, vp, vp, vp, u64, i32, vp, vp]
+    L.cszp2_container_index.argtypes = [vp, i32, vp, vp]
+    L.cszp2_version.restype = ctypes.c_char_p
+    return L
+
+
+_lib = _load()
+LIBRARY_PATH = _LIB_PATH
+EXPORTED = (
+    "cszp2_compress_bound", "cszp2_compress", "cszp2_compress_prepare", "cszp2_compress_encode",
+    "cszp2_decompress", "cszp2_read_header", "cszp2_compress_host", "cszp2_decompress_host",
+    "cszp2_container_index", "cszp2_version",
+)
+
+
+def version() -> str:
+    return _lib.cszp2_version().decode()
+
+
+def _stream(stream) -> int:
+    if stream is None:
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, torch.cuda.Stream):
+        return stream.cuda_stream
+    return int(stream)
+
+
+def _ptr(t: torch.Tensor | None):
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+def _check(fn: str, rc: int):
+    if rc != OK:
+        raise CszpError(fn, rc)
+
+
+def _need_cuda(*ts):
+    for t in ts:
+        if t is not None and not t.is_cuda:
+            raise ValueError("cszp2 operates on CUDA tensors only (no CPU fallback)")
+
+
+def compress_bound(n: int, dtype=torch.float32) -> int:
+    return int(_lib.cszp2_compress_bound(n, _DT[dtype] if isinstance(dtype, torch.dtype) else dtype))
+
+
+def compress(x: torch.Tensor, eb: float, eb_mode="abs", enc_mode="plain", out=None, out_bytes=None,
+             stream=None):
+    """Compress a contiguous CUDA f32/f64 tensor. Returns (stream buffer of
+    compress_bound bytes, device uint64-as-int64 tensor holding the stream's
+    byte count). Asynchronous on `stream` (default: torch's current stream)."""
+    _need_cuda(x, out, out_bytes)
+    x = x.contiguous().view(-1)
+    dt = _DT[x.dtype]
+    if out is None:
+        out = torch.empty(compress_bound(x.numel(), dt), dtype=torch.uint8, device=x.device)
+    if out_bytes is None:
+        out_bytes = torch.zeros(1, dtype=torch.int64, device=x.device)
+    rc = _lib.cszp2_compress(_ptr(x), x.numel(), dt, float(eb), _EB[eb_mode], _ENC[enc_mode],
+                             _ptr(out), _ptr(out_bytes), _stream(stream))
+    _check("cszp2_compress", rc)
+    return out, out_bytes
+
+
+def compress_prepare(x, eb, eb_mode, out, stream=None):
+    rc = _lib.cszp2_compress_prepare(_ptr(x), x.numel(), _DT[x.dtype], float(eb), _EB[eb_mode],
+                                     _ptr(out), _stream(stream))
+    _check("cszp2_compress_prepare", rc)
+
+
+def compress_encode(x, eb, eb_mode, enc_mode, out, out_bytes=None, stream=None):
+    rc = _lib.cszp2_compress_encode(_ptr(x), x.numel(), _DT[x.dtype], float(eb), _EB[eb_mode],
+                                    _ENC[enc_mode], _ptr(out), _ptr(out_bytes), _stream(stream))
+    _check("cszp2_compress_encode", rc)
+
+
+def decompress(cmp: torch.Tensor, n: int, dtype=torch.float32, out=None, status=None, stream=None):
+    """Decompress a device stream into n values. `status` (optional device
+    int32 tensor, zeroed by the caller) receives CSZP2_ERR_FORMAT/RANGE bits."""
+    _need_cuda(cmp, out, status)
+    if out is None:
+        out = torch.empty(n, dtype=dtype, device=cmp.device)
+    rc = _lib.cszp2_decompress(_ptr(cmp), _ptr(out), n, _DT[out.dtype], _ptr(status), _stream(stream))
+    _check("cszp2_decompress", rc)
+    return out
+
+
+def read_header(cmp: torch.Tensor, stream=None) -> dict:
+    _need_cuda(cmp)
+    h = Header()
+    _check("cszp2_read_header", _lib.cszp2_read_header(_ptr(cmp), ctypes.byref(h), _stream(stream)))
+    return h.as_dict()
+
+
+def compress_host(h_in: torch.Tensor, eb: float, eb_mode, enc_mode, d_in_work, d_out_work,
+                  h_out: torch.Tensor, stream=None) -> int:
+    """End-to-end from HOST memory: H2D, compress, D2H of the stream. Returns
+    the stream's byte count (synchronises)."""
+    nbytes = ctypes.c_uint64(0)
+    rc = _lib.cszp2_compress_host(_ptr(h_in), h_in.numel(), _DT[h_in.dtype], float(eb), _EB[eb_mode],
+                                  _ENC[enc_mode], _ptr(d_in_work), _ptr(d_out_work), _ptr(h_out),
+                                  h_out.numel(), ctypes.byref(nbytes), _stream(stream))
+    _check("cszp2_compress_host", rc)
+    return nbytes.value
+
+
+def decompress_host(h_cmp: torch.Tensor, cmp_bytes: int, d_cmp_work, d_out_work, h_out: torch.Tensor,
+                    status=None, stream=None):
+    rc = _lib.cszp2_decompress_host(_ptr(h_cmp), cmp_bytes, _ptr(d_cmp_work), _ptr(d_out_work),
+                                    _ptr(h_out), h_out.numel(), _DT[h_out.dtype], _ptr(status),
+                                    _stream(stream))
+    _check("cszp2_decompress_host", rc)
+    return h_out
+
+
+def container_index(sizes: torch.Tensor, out=None, stream=None):
+    """Exclusive scan of per-rank stream sizes (device int64[P]) -> int64[P+1]."""
+    _need_cuda(sizes, out)
+    if out is None:
+        out = torch.empty(sizes.numel() + 1, dtype=torch.int64, device=sizes.device)
+    _check("cszp2_container_index",
+           _lib.cszp2_container_index(_ptr(sizes), sizes.numel(), _ptr(out), _stream(stream)))
+    return out

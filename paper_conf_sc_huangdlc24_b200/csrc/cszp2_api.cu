@@ -1,0 +1,269 @@
+// cszp2_api.cu — C ABI (include/cszp2.h) over the sm_100a kernels in kernels.cuh.
+// Argument validation, stream geometry (FORMAT.md §2), tensor-map encoding and
+// launches. No compute happens on the host.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+#include <cuda_runtime.h>
+
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+
+#include "cszp2.h"
+#include "kernels.cuh"
+
+using namespace cszp2;
+
+namespace {
+
+inline cudaStream_t S(void *s) { return reinterpret_cast<cudaStream_t>(s); }
+
+Geom geometry(uint64_t n) {
+    Geom g;
+    g.n = n;
+    g.nb = (n + L - 1) / L;
+    g.nfull = n / L;
+    g.T = (g.nb + BPT - 1) / BPT;
+    g.O = roundup16(64 + 8 * g.T);
+    g.D = roundup16(g.O + g.nb);
+    return g;
+}
+
+bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+int wsize(int dtype) { return dtype == CSZP2_F32 ? 4 : (dtype == CSZP2_F64 ? 8 : 0); }
+
+PFN_cuTensorMapEncodeTiled_v12000 encoder() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) ==
+                cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+    });
+    return fn;
+}
+
+// Dense value side of a tile as a 2D tensor of 128-byte rows (one f32 block or
+// half an f64 block per row), box = 256 rows, 128-byte swizzle.
+int make_tmap(CUtensorMap *m, const void *base, int dtype, uint64_t nfull) {
+    std::memset(m, 0, sizeof(*m));
+    if (nfull == 0) return CSZP2_OK;  // kernels never touch the map
+    auto enc = encoder();
+    if (!enc) return CSZP2_ERR_CUDA;
+    const bool f32 = dtype == CSZP2_F32;
+    cuuint64_t dims[2] = {f32 ? 32ull : 16ull, f32 ? nfull : 2 * nfull};
+    cuuint64_t strides[1] = {128};
+    cuuint32_t box[2] = {f32 ? 32u : 16u, 256u};
+    cuuint32_t estr[2] = {1, 1};
+    CUresult r = enc(m, f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2,
+                     const_cast<void *>(base), dims, strides, box, estr,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS ? CSZP2_OK : CSZP2_ERR_CUDA;
+}
+
+template <typename K>
+int set_smem(K kernel, int bytes) {
+    return cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) ==
+                   cudaSuccess
+               ? CSZP2_OK
+               : CSZP2_ERR_CUDA;
+}
+
+int launch_status() { return cudaGetLastError() == cudaSuccess ? CSZP2_OK : CSZP2_ERR_CUDA; }
+
+int check_compress_args(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
+                        const void *d_out) {
+    if (!wsize(dtype) || !d_out || (!d_in && n)) return CSZP2_ERR_ARG;
+    if (eb_mode != CSZP2_EB_ABS && eb_mode != CSZP2_EB_REL) return CSZP2_ERR_ARG;
+    if (!(eb > 0.0) || !std::isfinite(eb)) return CSZP2_ERR_ARG;
+    if (!aligned16(d_out) || (n && !aligned16(d_in))) return CSZP2_ERR_ARG;
+    if (n > (1ull << 40)) return CSZP2_ERR_ARG;  // TMA row coordinates are int32
+    return CSZP2_OK;
+}
+
+template <typename T>
+int launch_minmax(const void *d_in, uint64_t n, double lambda, void *d_out, cudaStream_t st) {
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const uint64_t nvec = n / (16 / sizeof(T));
+    uint64_t want = (nvec + 255) / 256;
+    int grid = static_cast<int>(want < 1 ? 1 : (want > (uint64_t)sms * 8 ? (uint64_t)sms * 8 : want));
+    minmax_kernel<T><<<grid, 256, 0, st>>>(static_cast<const T *>(d_in), n, lambda,
+                                            static_cast<uint8_t *>(d_out));
+    return launch_status();
+}
+
+template <typename T, bool OUTLIER>
+int launch_compress(const void *d_in, const Geom &g, double eb, int eb_mode, int enc_mode,
+                    void *d_out, uint64_t *d_out_bytes, cudaStream_t st) {
+    static std::once_flag once;
+    static int attr_rc = CSZP2_OK;
+    constexpr int smem = compress_smem_bytes<T>();
+    std::call_once(once, [] { attr_rc = set_smem(compress_kernel<T, OUTLIER>, smem); });
+    if (attr_rc) return attr_rc;
+    CUtensorMap map;
+    int rc = make_tmap(&map, d_in, Traits<T>::DTYPE, g.nfull);
+    if (rc) return rc;
+    HdrStatic hs;
+    hs.word1 = 1u | (static_cast<uint32_t>(Traits<T>::DTYPE) << 8) |
+               (static_cast<uint32_t>(enc_mode) << 16) | (5u << 24);
+    hs.eb_mode = static_cast<uint32_t>(eb_mode);
+    hs.eb_user = eb;
+    const uint64_t grid = g.T ? g.T : 1;
+    compress_kernel<T, OUTLIER><<<static_cast<unsigned>(grid), NT, smem, st>>>(
+        map, static_cast<const T *>(d_in), g, eb, eb_mode == CSZP2_EB_REL ? 1 : 0,
+        static_cast<uint8_t *>(d_out), d_out_bytes, hs);
+    return launch_status();
+}
+
+template <typename T>
+int launch_decompress(const void *d_cmp, void *d_out, const Geom &g, int *d_status,
+                      cudaStream_t st) {
+    static std::once_flag once;
+    static int attr_rc = CSZP2_OK;
+    constexpr int smem = decompress_smem_bytes<T>();
+    std::call_once(once, [] { attr_rc = set_smem(decompress_kernel<T>, smem); });
+    if (attr_rc) return attr_rc;
+    CUtensorMap map;
+    int rc = make_tmap(&map, d_out, Traits<T>::DTYPE, g.nfull);
+    if (rc) return rc;
+    const uint64_t grid = g.T ? g.T : 1;
+    decompress_kernel<T><<<static_cast<unsigned>(grid), NT, smem, st>>>(
+        map, static_cast<const uint8_t *>(d_cmp), static_cast<T *>(d_out), g, d_status);
+    return launch_status();
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *cszp2_version(void) { return "cszp2 1.0 sm_100a"; }
+
+uint64_t cszp2_compress_bound(uint64_t n, int dtype) {
+    if (!wsize(dtype)) return 0;
+    Geom g = geometry(n);
+    return roundup16(g.D + static_cast<uint64_t>(4 * L) * g.nb);
+}
+
+int cszp2_compress_prepare(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
+                           void *d_out, void *stream) {
+    int rc = check_compress_args(d_in, n, dtype, eb, eb_mode, d_out);
+    if (rc) return rc;
+    Geom g = geometry(n);
+    if (cudaMemsetAsync(d_out, 0, g.O, S(stream)) != cudaSuccess) return CSZP2_ERR_CUDA;
+    if (eb_mode == CSZP2_EB_REL)
+        return dtype == CSZP2_F32 ? launch_minmax<float>(d_in, n, eb, d_out, S(stream))
+                                  : launch_minmax<double>(d_in, n, eb, d_out, S(stream));
+    return CSZP2_OK;
+}
+
+int cszp2_compress_encode(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
+                          int enc_mode, void *d_out, uint64_t *d_out_bytes, void *stream) {
+    int rc = check_compress_args(d_in, n, dtype, eb, eb_mode, d_out);
+    if (rc) return rc;
+    if (enc_mode != CSZP2_ENC_PLAIN && enc_mode != CSZP2_ENC_OUTLIER) return CSZP2_ERR_ARG;
+    Geom g = geometry(n);
+    if (dtype == CSZP2_F32)
+        return enc_mode == CSZP2_ENC_OUTLIER
+                   ? launch_compress<float, true>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, S(stream))
+                   : launch_compress<float, false>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, S(stream));
+    return enc_mode == CSZP2_ENC_OUTLIER
+               ? launch_compress<double, true>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, S(stream))
+               : launch_compress<double, false>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, S(stream));
+}
+
+int cszp2_compress(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode, int enc_mode,
+                   void *d_out, uint64_t *d_out_bytes, void *stream) {
+    if (enc_mode != CSZP2_ENC_PLAIN && enc_mode != CSZP2_ENC_OUTLIER) return CSZP2_ERR_ARG;
+    int rc = cszp2_compress_prepare(d_in, n, dtype, eb, eb_mode, d_out, stream);
+    if (rc) return rc;
+    return cszp2_compress_encode(d_in, n, dtype, eb, eb_mode, enc_mode, d_out, d_out_bytes, stream);
+}
+
+int cszp2_decompress(const void *d_cmp, void *d_out, uint64_t n, int dtype, int *d_status,
+                     void *stream) {
+    if (!wsize(dtype) || !d_cmp || (!d_out && n)) return CSZP2_ERR_ARG;
+    if (!aligned16(d_cmp) || (n && !aligned16(d_out))) return CSZP2_ERR_ARG;
+    if (n > (1ull << 40)) return CSZP2_ERR_ARG;
+    Geom g = geometry(n);
+    return dtype == CSZP2_F32 ? launch_decompress<float>(d_cmp, d_out, g, d_status, S(stream))
+                              : launch_decompress<double>(d_cmp, d_out, g, d_status, S(stream));
+}
+
+int cszp2_read_header(const void *d_cmp, cszp2_header *h, void *stream) {
+    if (!d_cmp || !h) return CSZP2_ERR_ARG;
+    uint8_t raw[64];
+    if (cudaMemcpyAsync(raw, d_cmp, 64, cudaMemcpyDeviceToHost, S(stream)) != cudaSuccess ||
+        cudaStreamSynchronize(S(stream)) != cudaSuccess)
+        return CSZP2_ERR_CUDA;
+    std::memcpy(&h->magic, raw + 0, 4);
+    h->version = raw[4];
+    h->dtype = raw[5];
+    h->enc_mode = raw[6];
+    h->log2L = raw[7];
+    h->eb_mode = raw[8];
+    h->status = raw[9];
+    std::memcpy(&h->blocks_per_tile, raw + 10, 2);
+    std::memcpy(&h->n, raw + 16, 8);
+    std::memcpy(&h->eb, raw + 24, 8);
+    std::memcpy(&h->eb_abs, raw + 32, 8);
+    std::memcpy(&h->payload_bytes, raw + 40, 8);
+    std::memcpy(&h->total_bytes, raw + 48, 8);
+    return CSZP2_OK;
+}
+
+int cszp2_compress_host(const void *h_in, uint64_t n, int dtype, double eb, int eb_mode,
+                        int enc_mode, void *d_in_work, void *d_out_work, void *h_out,
+                        uint64_t h_out_cap, uint64_t *h_out_bytes, void *stream) {
+    if (!h_out || !h_out_bytes || (!h_in && n)) return CSZP2_ERR_ARG;
+    const int w = wsize(dtype);
+    if (!w) return CSZP2_ERR_ARG;
+    if (n && cudaMemcpyAsync(d_in_work, h_in, n * w, cudaMemcpyHostToDevice, S(stream)) != cudaSuccess)
+        return CSZP2_ERR_CUDA;
+    int rc = cszp2_compress(d_in_work, n, dtype, eb, eb_mode, enc_mode, d_out_work, nullptr, stream);
+    if (rc) return rc;
+    uint64_t total = 0;  // the stream's own header holds its size (FORMAT.md §3)
+    if (cudaMemcpyAsync(&total, static_cast<uint8_t *>(d_out_work) + 48, 8, cudaMemcpyDeviceToHost,
+                        S(stream)) != cudaSuccess ||
+        cudaStreamSynchronize(S(stream)) != cudaSuccess)
+        return CSZP2_ERR_CUDA;
+    if (total > h_out_cap) return CSZP2_ERR_ARG;
+    if (cudaMemcpyAsync(h_out, d_out_work, total, cudaMemcpyDeviceToHost, S(stream)) != cudaSuccess ||
+        cudaStreamSynchronize(S(stream)) != cudaSuccess)
+        return CSZP2_ERR_CUDA;
+    *h_out_bytes = total;
+    return CSZP2_OK;
+}
+
+int cszp2_decompress_host(const void *h_cmp, uint64_t cmp_bytes, void *d_cmp_work,
+                          void *d_out_work, void *h_out, uint64_t n, int dtype, int *d_status,
+                          void *stream) {
+    const int w = wsize(dtype);
+    if (!w || !h_cmp || !d_cmp_work || (n && (!h_out || !d_out_work))) return CSZP2_ERR_ARG;
+    if (cudaMemcpyAsync(d_cmp_work, h_cmp, cmp_bytes, cudaMemcpyHostToDevice, S(stream)) != cudaSuccess)
+        return CSZP2_ERR_CUDA;
+    int rc = cszp2_decompress(d_cmp_work, d_out_work, n, dtype, d_status, stream);
+    if (rc) return rc;
+    if (n && cudaMemcpyAsync(h_out, d_out_work, n * w, cudaMemcpyDeviceToHost, S(stream)) != cudaSuccess)
+        return CSZP2_ERR_CUDA;
+    int st = 0;
+    if (d_status && cudaMemcpyAsync(&st, d_status, 4, cudaMemcpyDeviceToHost, S(stream)) != cudaSuccess)
+        return CSZP2_ERR_CUDA;
+    if (cudaStreamSynchronize(S(stream)) != cudaSuccess) return CSZP2_ERR_CUDA;
+    return st;
+}
+
+int cszp2_container_index(const uint64_t *d_sizes, int nparts, uint64_t *d_offsets,
+                          void *stream) {
+    if (!d_sizes || !d_offsets || nparts < 1) return CSZP2_ERR_ARG;
+    container_index_kernel<<<1, 32, 0, S(stream)>>>(d_sizes, nparts, d_offsets);
+    return launch_status();
+}
+
+}  // extern "C"

@@ -1,0 +1,711 @@
+// kernels.cuh — sm_100a kernels of the cuSZp2 hot path (FORMAT.md; PAPER.md).
+//
+//   minmax_kernel      REL -> ABS: grid-wide exact min/max, eb_abs = λ·(max−min)
+//   compress_kernel    ❶ pre-quantization → in-block 1D Lorenzo → ❷ Plain/Outlier
+//                      FLE → ❸ decoupled-lookback exclusive scan → ❹ concatenation,
+//                      one fused pass (Fig 4)
+//   decompress_kernel  ❸ (O(1) from the persisted tile index) → ❹ → ❷⁻¹ → ❶⁻¹
+//
+// B200 design: one CTA = one tile of 256 blocks (8192 f32 values);
+// one thread = one 32-value block (block-level data parallelism). Tiles move
+// between HBM and shared memory with TMA: 2D tensor maps with 128-byte swizzle for
+// the dense value side (so thread-per-block 16-byte shared accesses are
+// bank-conflict free), 1D bulk copies for the byte-granular compressed side.
+// Bit planes are packed/unpacked with add.cc/addc carry chains (2 ops per bit).
+#pragma once
+#include <cstdint>
+#include <type_traits>
+#include <cuda.h>
+
+#include "ptx.cuh"
+
+namespace cszp2 {
+
+constexpr int L = 32;      // values per block
+constexpr int BPT = 256;   // blocks per tile (FORMAT.md §1)
+constexpr int NT = 256;    // threads per CTA: one block per thread
+constexpr uint32_t MAGIC = 0x325A5343u;
+constexpr uint64_t FLAG_A = 1ull << 62;   // lookback: aggregate available
+constexpr uint64_t FLAG_P = 2ull << 62;   // lookback: inclusive prefix available
+constexpr uint64_t VAL_MASK = (1ull << 62) - 1;
+constexpr int ST_RANGE = 3;
+constexpr int ST_FORMAT = 4;
+
+struct Geom {
+    uint64_t n;      // values
+    uint64_t nb;     // blocks = ceil(n / L)
+    uint64_t nfull;  // blocks with all L values = n / L
+    uint64_t T;      // tiles
+    uint64_t O;      // offset-byte region start
+    uint64_t D;      // payload region start
+};
+
+__host__ __device__ inline uint64_t roundup16(uint64_t v) { return (v + 15) & ~uint64_t(15); }
+
+template <typename T>
+struct Traits;
+template <>
+struct Traits<float> {
+    static constexpr int ROWS = 1;  // 128-byte TMA rows per block
+    static constexpr int TILE_BYTES = BPT * L * 4;
+    static constexpr int DTYPE = 0;
+};
+template <>
+struct Traits<double> {
+    static constexpr int ROWS = 2;
+    static constexpr int TILE_BYTES = BPT * L * 8;
+    static constexpr int DTYPE = 1;
+};
+
+// ------------------------------------------------------------------ arithmetic contract
+// FORMAT.md §6.2-6.3 / §6.6: RN multiply (no FMA), round-half-even conversion.
+struct ConstsF {
+    float inv, s;
+    bool ok;
+};
+struct ConstsD {
+    double inv, s;
+    bool ok;
+};
+__device__ __forceinline__ ConstsF make_consts(double eb, float *) {
+    ConstsF c;
+    c.inv = __double2float_rn(__ddiv_rn(1.0, __dmul_rn(2.0, eb)));
+    c.s = __double2float_rn(__dmul_rn(2.0, eb));
+    c.ok = (eb > 0.0) && isfinite(eb) && (c.inv > 0.0f) && isfinite(c.inv) && (c.s > 0.0f) &&
+           isfinite(c.s);
+    return c;
+}
+__device__ __forceinline__ ConstsD make_consts(double eb, double *) {
+    ConstsD c;
+    c.inv = __ddiv_rn(1.0, __dmul_rn(2.0, eb));
+    c.s = __dmul_rn(2.0, eb);
+    c.ok = (eb > 0.0) && isfinite(eb) && (c.inv > 0.0) && isfinite(c.inv) && (c.s > 0.0) &&
+           isfinite(c.s);
+    return c;
+}
+__device__ __forceinline__ int quantize(float x, float inv, bool &bad) {
+    float t = __fmul_rn(x, inv);
+    bad |= !(fabsf(t) <= 1073741760.0f);  // also true for NaN
+    return __float2int_rn(t);
+}
+__device__ __forceinline__ int quantize(double x, double inv, bool &bad) {
+    double t = __dmul_rn(x, inv);
+    bad |= !(fabs(t) <= 1073741823.0);
+    return __double2int_rn(t);
+}
+__device__ __forceinline__ float dequantize(int q, float s) { return __fmul_rn(__int2float_rn(q), s); }
+__device__ __forceinline__ double dequantize(int q, double s) {
+    return __dmul_rn(__int2double_rn(q), s);
+}
+
+// ------------------------------------------------------------------ swizzled tile access
+// TMA SWIZZLE_128B: the 16-byte chunk c of 128-byte row r lives at chunk c ^ (r & 7).
+__device__ __forceinline__ uint32_t swz(uint32_t row, uint32_t chunk) {
+    return row * 128u + ((chunk ^ (row & 7u)) << 4);
+}
+__device__ __forceinline__ void load_block(const uint8_t *tile, uint32_t r, float (&x)[L]) {
+#pragma unroll
+    for (int c = 0; c < 8; c++) {
+        float4 v = *reinterpret_cast<const float4 *>(tile + swz(r, c));
+        x[4 * c + 0] = v.x;
+        x[4 * c + 1] = v.y;
+        x[4 * c + 2] = v.z;
+        x[4 * c + 3] = v.w;
+    }
+}
+__device__ __forceinline__ void load_block(const uint8_t *tile, uint32_t r, double (&x)[L]) {
+#pragma unroll
+    for (int h = 0; h < 2; h++)
+#pragma unroll
+        for (int c = 0; c < 8; c++) {
+            double2 v = *reinterpret_cast<const double2 *>(tile + swz(2 * r + h, c));
+            x[16 * h + 2 * c + 0] = v.x;
+            x[16 * h + 2 * c + 1] = v.y;
+        }
+}
+__device__ __forceinline__ void store_block(uint8_t *tile, uint32_t r, const float (&x)[L]) {
+#pragma unroll
+    for (int c = 0; c < 8; c++)
+        *reinterpret_cast<float4 *>(tile + swz(r, c)) =
+            make_float4(x[4 * c], x[4 * c + 1], x[4 * c + 2], x[4 * c + 3]);
+}
+__device__ __forceinline__ void store_block(uint8_t *tile, uint32_t r, const double (&x)[L]) {
+#pragma unroll
+    for (int h = 0; h < 2; h++)
+#pragma unroll
+        for (int c = 0; c < 8; c++)
+            *reinterpret_cast<double2 *>(tile + swz(2 * r + h, c)) =
+                make_double2(x[16 * h + 2 * c], x[16 * h + 2 * c + 1]);
+}
+
+// ------------------------------------------------------------------ byte-granular smem access
+__device__ __forceinline__ void st_u32_unaligned(uint8_t *p, uint32_t w) {
+    if ((reinterpret_cast<uintptr_t>(p) & 3u) == 0) {
+        *reinterpret_cast<uint32_t *>(p) = w;
+    } else {
+        p[0] = static_cast<uint8_t>(w);
+        p[1] = static_cast<uint8_t>(w >> 8);
+        p[2] = static_cast<uint8_t>(w >> 16);
+        p[3] = static_cast<uint8_t>(w >> 24);
+    }
+}
+__device__ __forceinline__ uint32_t ld_u32_unaligned(const uint8_t *base, uint32_t pos) {
+    const uint32_t *w = reinterpret_cast<const uint32_t *>(base + (pos & ~3u));
+    return __funnelshift_r(w[0], w[1], 8u * (pos & 3u));
+}
+
+// ------------------------------------------------------------------ scans
+__device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+// CTA-wide exclusive scan of one u32 per thread (NT = 256). Returns the
+// exclusive prefix; *total receives the sum. Contains two __syncthreads.
+__device__ __forceinline__ uint32_t cta_exclusive_scan(uint32_t v, uint32_t *s_warp,
+                                                       uint32_t *total) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    uint32_t inc = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
+    }
+    if (lane == 31) s_warp[warp] = inc;
+    __syncthreads();
+    uint32_t base = 0, tot = 0;
+#pragma unroll
+    for (int w = 0; w < NT / 32; w++) {
+        uint32_t s = s_warp[w];
+        base += (w < warp) ? s : 0u;
+        tot += s;
+    }
+    *total = tot;
+    __syncthreads();
+    return base + inc - v;
+}
+
+// ❸ Decoupled lookback (Fig 13; after Merrill & Garland [25]).
+// Executed by one full warp. Tile t publishes (A | aggregate), then walks back
+// over its predecessors' descriptors 32 at a time, summing aggregates until it
+// meets an inclusive prefix (P); then publishes (P | inclusive). The final
+// descriptors ARE the stream's tile index (FORMAT.md §2). Returns the
+// exclusive prefix of tile t.
+__device__ __forceinline__ uint64_t lookback(uint64_t *index, uint64_t t, uint64_t agg) {
+    const int lane = threadIdx.x & 31;
+    if (t == 0) {
+        if (lane == 0) st_release_u64(&index[0], FLAG_P | agg);
+        return 0;
+    }
+    if (lane == 0) st_release_u64(&index[t], FLAG_A | agg);
+    uint64_t excl = 0;
+    int64_t j = static_cast<int64_t>(t) - 1;
+    while (true) {
+        const int64_t idx = j - lane;
+        uint64_t d = FLAG_P;  // virtual P|0 before tile 0
+        if (idx >= 0) {
+            d = ld_acquire_u64(&index[idx]);
+            while ((d >> 62) == 0) {  // Waiting: spin until published
+                __nanosleep(20);
+                d = ld_acquire_u64(&index[idx]);
+            }
+        }
+        const unsigned pmask = __ballot_sync(0xffffffffu, (d >> 62) == 2);
+        uint64_t v = d & VAL_MASK;
+        if (pmask) {
+            const int p = __ffs(pmask) - 1;  // nearest predecessor with a prefix
+            excl += warp_sum_u64(lane <= p ? v : 0);
+            break;
+        }
+        excl += warp_sum_u64(v);
+        j -= 32;
+    }
+    if (lane == 0) st_release_u64(&index[t], FLAG_P | (excl + agg));
+    return excl;
+}
+
+// ------------------------------------------------------------------ REL: min/max
+__device__ __forceinline__ uint32_t sortable(float x) {
+    uint32_t u = __float_as_uint(x);
+    return u ^ ((u & 0x80000000u) ? 0xFFFFFFFFu : 0x80000000u);
+}
+__device__ __forceinline__ float unsortable(uint32_t u) {
+    return __uint_as_float(u ^ ((u & 0x80000000u) ? 0x80000000u : 0xFFFFFFFFu));
+}
+__device__ __forceinline__ unsigned long long sortable(double x) {
+    unsigned long long u = __double_as_longlong(x);
+    return u ^ ((u >> 63) ? 0xFFFFFFFFFFFFFFFFull : 0x8000000000000000ull);
+}
+__device__ __forceinline__ double unsortable(unsigned long long u) {
+    return __longlong_as_double(u ^ ((u >> 63) ? 0x8000000000000000ull : 0xFFFFFFFFFFFFFFFFull));
+}
+
+// Header scratch while the REL reduction runs (the memset zeroed it; the last
+// CTA restores zeros): [40] sortable max, [48] ~sortable min, [56] u32 CTA counter.
+template <typename T>
+__global__ void __launch_bounds__(256) minmax_kernel(const T *__restrict__ in, uint64_t n,
+                                                     double lambda, uint8_t *__restrict__ hdr) {
+    using V = typename std::conditional<sizeof(T) == 4, float4, double2>::type;
+    constexpr int PER = 16 / sizeof(T);
+    T mn = INFINITY, mx = -INFINITY;
+    const uint64_t nvec = n / PER;
+    const V *vin = reinterpret_cast<const V *>(in);
+    const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
+    uint64_t i = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+    // 4-way unrolled grid-stride loop (loads in flight before the min/max)
+    for (; i + 3 * stride < nvec; i += 4 * stride) {
+        V v[4];
+#pragma unroll
+        for (int u = 0; u < 4; u++) v[u] = __ldcs(vin + i + u * stride);
+#pragma unroll
+        for (int u = 0; u < 4; u++) {
+            const T *e = reinterpret_cast<const T *>(&v[u]);
+#pragma unroll
+            for (int k = 0; k < PER; k++) {
+                mn = fmin(mn, e[k]);
+                mx = fmax(mx, e[k]);
+            }
+        }
+    }
+    for (; i < nvec; i += stride) {
+        V v = __ldcs(vin + i);
+        const T *e = reinterpret_cast<const T *>(&v);
+#pragma unroll
+        for (int k = 0; k < PER; k++) {
+            mn = fmin(mn, e[k]);
+            mx = fmax(mx, e[k]);
+        }
+    }
+    if (blockIdx.x == 0 && threadIdx.x < n - nvec * PER) {
+        T e = in[nvec * PER + threadIdx.x];
+        mn = fmin(mn, e);
+        mx = fmax(mx, e);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        mn = fmin(mn, __shfl_xor_sync(0xffffffffu, mn, o));
+        mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    }
+    __shared__ T s_mn[8], s_mx[8];
+    __shared__ bool s_last;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    if (lane == 0) {
+        s_mn[warp] = mn;
+        s_mx[warp] = mx;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int w = 1; w < (int)(blockDim.x / 32); w++) {
+            mn = fmin(mn, s_mn[w]);
+            mx = fmax(mx, s_mx[w]);
+        }
+        if (mn <= mx) {  // at least one non-NaN value
+            if (sizeof(T) == 4) {
+                atomicMax(reinterpret_cast<unsigned *>(hdr + 40), (unsigned)sortable(mx));
+                atomicMax(reinterpret_cast<unsigned *>(hdr + 48), ~(unsigned)sortable(mn));
+            } else {
+                atomicMax(reinterpret_cast<unsigned long long *>(hdr + 40),
+                          (unsigned long long)sortable(mx));
+                atomicMax(reinterpret_cast<unsigned long long *>(hdr + 48),
+                          ~(unsigned long long)sortable(mn));
+            }
+        }
+        __threadfence();
+        unsigned prev = atomicAdd(reinterpret_cast<unsigned *>(hdr + 56), 1u);
+        s_last = (prev == gridDim.x - 1);
+    }
+    __syncthreads();
+    if (s_last && threadIdx.x == 0) {
+        __threadfence();
+        double r = 0.0;
+        if (sizeof(T) == 4) {
+            unsigned emx = atomicAdd(reinterpret_cast<unsigned *>(hdr + 40), 0u);
+            unsigned emn = ~atomicAdd(reinterpret_cast<unsigned *>(hdr + 48), 0u);
+            if (emx != 0u)
+                r = __dsub_rn((double)unsortable(emx), (double)unsortable(emn));
+        } else {
+            unsigned long long emx =
+                atomicAdd(reinterpret_cast<unsigned long long *>(hdr + 40), 0ull);
+            unsigned long long emn =
+                ~atomicAdd(reinterpret_cast<unsigned long long *>(hdr + 48), 0ull);
+            if (emx != 0ull) r = __dsub_rn(unsortable(emx), unsortable(emn));
+        }
+        const double eb_abs = (r == 0.0) ? lambda : __dmul_rn(lambda, r);
+        *reinterpret_cast<double *>(hdr + 32) = eb_abs;
+        reinterpret_cast<unsigned long long *>(hdr + 40)[0] = 0ull;
+        reinterpret_cast<unsigned long long *>(hdr + 40)[1] = 0ull;
+        reinterpret_cast<unsigned long long *>(hdr + 40)[2] = 0ull;
+    }
+}
+
+// ------------------------------------------------------------------ compression
+struct HdrStatic {
+    uint32_t word1;    // header bytes 4..7: version, dtype, enc_mode, log2L
+    uint32_t eb_mode;  // header byte 8
+    double eb_user;    // header bytes 24..31
+};
+
+template <typename T>
+constexpr int compress_smem_bytes() {
+    return Traits<T>::TILE_BYTES + 1024 + 128;
+}
+
+template <typename T, bool OUTLIER>
+__global__ void __launch_bounds__(NT) compress_kernel(const __grid_constant__ CUtensorMap tmap,
+                                                      const T *__restrict__ in, const Geom g,
+                                                      const double eb_abs_arg,
+                                                      const int eb_from_header,
+                                                      uint8_t *__restrict__ out,
+                                                      uint64_t *__restrict__ d_out_bytes,
+                                                      const HdrStatic hs) {
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t *tile = reinterpret_cast<uint8_t *>(
+        (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    __shared__ uint64_t s_bar;
+    __shared__ uint32_t s_ticket;
+    __shared__ uint32_t s_warp[NT / 32];
+    __shared__ uint64_t s_tile_excl;
+
+    const int tid = threadIdx.x;
+    const uint64_t T_eff = g.T ? g.T : 1;
+
+    if (tid == 0) {
+        // dynamic tile id: tiles are handed out in order, so every predecessor a
+        // lookback waits for is already resident (forward progress)
+        s_ticket = atomicAdd(reinterpret_cast<unsigned *>(out + 56), 1u);
+        mbar_init(&s_bar, 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    const uint64_t t = s_ticket;
+    const uint64_t b0 = t * BPT;
+    const bool has_rows = b0 < g.nfull;
+    if (tid == 0 && has_rows) {
+        if (Traits<T>::ROWS == 1) {
+            mbar_expect_tx(&s_bar, BPT * 128);
+            tma_load_2d(tile, &tmap, 0, static_cast<int>(b0), &s_bar);
+        } else {
+            const bool second = (b0 + BPT / 2) < g.nfull;
+            mbar_expect_tx(&s_bar, second ? 2 * BPT * 128 : BPT * 128);
+            tma_load_2d(tile, &tmap, 0, static_cast<int>(2 * b0), &s_bar);
+            if (second)
+                tma_load_2d(tile + BPT * 128, &tmap, 0, static_cast<int>(2 * b0 + BPT), &s_bar);
+        }
+    }
+
+    // constants of the arithmetic contract (FORMAT.md §6.2)
+    const double eb_abs =
+        eb_from_header ? *reinterpret_cast<const volatile double *>(out + 32) : eb_abs_arg;
+    const auto K = make_consts(eb_abs, static_cast<T *>(nullptr));
+
+    const uint64_t b = b0 + tid;
+    const bool active = b < g.nb;
+    const bool full = b < g.nfull;
+
+    if (has_rows) mbar_wait(&s_bar, 0);
+
+    // ---- load the block's 32 values
+    T x[L];
+    uint32_t valid = L;
+    if (full) {
+        load_block(tile, tid, x);
+    } else {
+        valid = active ? static_cast<uint32_t>(g.n - b * L) : 0u;
+#pragma unroll
+        for (int i = 0; i < L; i++) x[i] = (i < (int)valid) ? in[b * L + i] : T(0);
+    }
+
+    // ---- ❶ pre-quantization + in-block first-order difference
+    bool bad = false;
+    int q[L];
+#pragma unroll
+    for (int i = 0; i < L; i++) q[i] = quantize(x[i], K.inv, bad);
+    if (!full) {  // tail block: q_i = q_{i-1} past n (FORMAT.md §6.4)
+#pragma unroll
+        for (int i = 1; i < L; i++)
+            if (i >= (int)valid) q[i] = q[i - 1];
+    }
+    uint32_t a[L];
+    uint32_t sign = 0, or_rest = 0;
+#pragma unroll
+    for (int i = 0; i < L; i++) {
+        const int d = q[i] - (i ? q[i - 1] : 0);
+        a[i] = static_cast<uint32_t>(d < 0 ? -d : d);
+        sign |= static_cast<uint32_t>(d < 0) << i;
+        if (i) or_rest |= a[i];
+    }
+
+    // ---- ❷ fixed lengths and the fine-tuned Plain/Outlier selection
+    const int fl_p = 32 - __clz(or_rest | a[0]);
+    uint32_t size = fl_p ? 4u * (1u + fl_p) : 0u;
+    uint32_t obyte = static_cast<uint32_t>(fl_p);
+    int fl = fl_p, nob = 0;
+    if (OUTLIER) {
+        const int fl_o = 32 - __clz(or_rest);
+        const int ob = max(1, (32 - __clz(a[0]) + 7) >> 3);
+        const uint32_t size_o = 4u + ob + 4u * fl_o;
+        if (size_o < size) {
+            size = size_o;
+            obyte = 0x80u | (static_cast<uint32_t>(ob - 1) << 5) | static_cast<uint32_t>(fl_o);
+            fl = fl_o;
+            nob = ob;
+        }
+    }
+    if (!active) {
+        size = 0;
+        bad = false;
+    }
+    if (!K.ok) bad = true;
+
+    // ---- ❸ intra-tile scan + decoupled lookback across tiles
+    const bool any_bad = __syncthreads_or(bad);
+    uint32_t agg;
+    const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg);
+    if (tid < 32) {
+        if (any_bad && tid == 0)  // status before the descriptor is released
+            atomicOr(reinterpret_cast<unsigned *>(out + 8), static_cast<unsigned>(ST_RANGE) << 8);
+        uint64_t excl = 0;
+        if (g.T) excl = lookback(reinterpret_cast<uint64_t *>(out + 64), t, agg);
+        if (tid == 0) s_tile_excl = excl;
+    }
+
+    // ---- ❹ concatenation: offset byte straight to global, payload staged in smem
+    if (active) out[g.O + b] = static_cast<uint8_t>(obyte);
+    __syncthreads();  // s_tile_excl visible; every thread is done reading `tile`
+    const uint64_t tile_excl = s_tile_excl;
+    const uint64_t dst0 = g.D + tile_excl;
+    const uint32_t phase = static_cast<uint32_t>(dst0 & 15u);
+    if (size) {
+        uint8_t *p = tile + phase + my_excl;
+        st_u32_unaligned(p, sign);
+        p += 4;
+        if (OUTLIER && nob) {
+            for (int j = 0; j < nob; j++) p[j] = static_cast<uint8_t>(a[0] >> (8 * j));
+            p += nob;
+            a[0] = 0;  // the outlier slot of every plane is 0
+        }
+        if (fl) {
+            const int sh = 32 - fl;
+#pragma unroll
+            for (int i = 0; i < L; i++) a[i] <<= sh;
+            for (int k = fl - 1; k >= 0; k--) {  // planes top-down, 2 ops per bit
+                uint32_t w = 0;
+#pragma unroll
+                for (int i = L - 1; i >= 0; i--) shift_bit_into(a[i], w);
+                st_u32_unaligned(p + 4 * k, w);
+            }
+        }
+    }
+    fence_proxy_async_smem();
+    __syncthreads();
+
+    const uint64_t dst1 = dst0 + agg;
+    const uint64_t m0 = roundup16(dst0), m1 = dst1 & ~uint64_t(15);
+    if (m0 < m1) {
+        if (tid == 0) {
+            bulk_store(out + m0, tile + (m0 - (dst0 & ~uint64_t(15))), static_cast<uint32_t>(m1 - m0));
+            bulk_commit();
+        }
+        if (tid >= 32 && tid < 48) {  // unaligned head bytes
+            const uint64_t o = dst0 + (tid - 32);
+            if (o < m0) out[o] = tile[phase + (o - dst0)];
+        }
+        if (tid >= 64 && tid < 80) {  // unaligned tail bytes
+            const uint64_t o = m1 + (tid - 64);
+            if (o < dst1) out[o] = tile[phase + (o - dst0)];
+        }
+    } else if (tid >= 96 && tid < 128) {  // whole tile payload < 32 bytes
+        const uint64_t o = dst0 + (tid - 96);
+        if (o < dst1) out[o] = tile[phase + (o - dst0)];
+    }
+
+    if (t == T_eff - 1) {  // last tile: pads, header, d_out_bytes
+        if (tid >= 128 && tid < 144) {  // zero pad after the payload
+            const uint64_t o = dst1 + (tid - 128);
+            if (o < roundup16(dst1)) out[o] = 0;
+        }
+        if (tid >= 160 && tid < 176) {  // zero pad after the offset bytes
+            const uint64_t o = g.O + g.nb + (tid - 160);
+            if (o < g.D) out[o] = 0;
+        }
+        if (tid == 0) {
+            const uint32_t w8 = ld_acquire_u32(reinterpret_cast<const uint32_t *>(out + 8));
+            const uint32_t status = (w8 >> 8) & 0xFFu;
+            const uint64_t pb = status ? 0 : tile_excl + agg;
+            const uint64_t total = roundup16(g.D + pb);
+            uint64_t *h = reinterpret_cast<uint64_t *>(out);
+            h[0] = MAGIC | (static_cast<uint64_t>(hs.word1) << 32);
+            h[1] = hs.eb_mode | (status << 8) | (static_cast<uint64_t>(BPT) << 16);
+            h[2] = g.n;
+            h[3] = static_cast<uint64_t>(__double_as_longlong(hs.eb_user));
+            h[4] = static_cast<uint64_t>(__double_as_longlong(eb_abs));
+            h[5] = pb;
+            h[6] = total;
+            h[7] = 0;
+            if (d_out_bytes) *d_out_bytes = total;
+        }
+    }
+    if (tid == 0 && m0 < m1) bulk_wait0();
+}
+
+// ------------------------------------------------------------------ decompression
+template <typename T>
+constexpr int decompress_smem_bytes() {
+    return Traits<T>::TILE_BYTES + BPT * 4 * L + 64 + 1024 + 128;
+}
+
+template <typename T>
+__global__ void __launch_bounds__(NT) decompress_kernel(const __grid_constant__ CUtensorMap tmap,
+                                                        const uint8_t *__restrict__ cmp,
+                                                        T *__restrict__ out, const Geom g,
+                                                        int *__restrict__ d_status) {
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t *ostage = reinterpret_cast<uint8_t *>(
+        (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint8_t *pbuf = ostage + Traits<T>::TILE_BYTES;
+    __shared__ uint64_t s_bar;
+    __shared__ uint32_t s_warp[NT / 32];
+    __shared__ uint64_t s_excl, s_bytes;
+    __shared__ double s_eb;
+    __shared__ int s_err;
+
+    const int tid = threadIdx.x;
+    const uint64_t t = blockIdx.x;
+    if (tid == 0) {
+        // header checks (FORMAT.md §3) — every CTA reads the 64 L2-resident bytes
+        const uint64_t *h = reinterpret_cast<const uint64_t *>(cmp);
+        const uint64_t h0 = h[0], h1 = h[1];
+        int err = 0;
+        const uint32_t want1 = 1u | (static_cast<uint32_t>(Traits<T>::DTYPE) << 8) | (5u << 24);
+        if ((h0 & 0xFFFFFFFFu) != MAGIC || ((h0 >> 32) & 0xFF00FFFFu) != want1 ||
+            ((h1 >> 16) & 0xFFFFu) != BPT || h[2] != g.n)
+            err = ST_FORMAT;
+        else if (((h1 >> 8) & 0xFF) != 0)
+            err = ((h1 >> 8) & 0xFF) == ST_RANGE ? ST_RANGE : ST_FORMAT;
+        const uint64_t pb = h[5];
+        if (!err && h[6] != roundup16(g.D + pb)) err = ST_FORMAT;
+        uint64_t excl = 0, incl = 0;
+        if (!err && t < g.T) {
+            const uint64_t *index = h + 8;
+            const uint64_t dp = t ? index[t - 1] : FLAG_P;
+            const uint64_t di = index[t];
+            excl = dp & VAL_MASK;
+            incl = di & VAL_MASK;
+            if ((dp >> 62) != 2 || (di >> 62) != 2 || incl < excl || incl > pb ||
+                incl - excl > static_cast<uint64_t>(BPT) * 4 * L)
+                err = ST_FORMAT;
+        }
+        s_eb = __longlong_as_double(static_cast<long long>(h[4]));
+        s_excl = excl;
+        s_bytes = incl - excl;
+        s_err = err;
+        mbar_init(&s_bar, 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    if (s_err || t >= g.T) {
+        if (tid == 0 && s_err && d_status) atomicOr(d_status, s_err);
+        return;
+    }
+    const uint64_t excl = s_excl;
+    const uint32_t bytes = static_cast<uint32_t>(s_bytes);
+    const uint64_t src0 = (g.D + excl) & ~uint64_t(15);
+    const uint32_t phase = static_cast<uint32_t>((g.D + excl) & 15u);
+    if (tid == 0 && bytes) {  // ❸ located in O(1): fetch the tile's payload bytes
+        const uint32_t len = static_cast<uint32_t>(roundup16(g.D + excl + bytes) - src0);
+        mbar_expect_tx(&s_bar, len);
+        bulk_load(pbuf, cmp + src0, len, &s_bar);
+    }
+
+    const uint64_t b = t * BPT + tid;
+    const bool active = b < g.nb;
+    const uint32_t obyte = active ? cmp[g.O + b] : 0u;
+    const uint32_t fl = obyte & 31u;
+    const bool is_o = (obyte & 0x80u) != 0;
+    const uint32_t nob = is_o ? ((obyte >> 5) & 3u) + 1u : 0u;
+    bool bad = (!is_o && (obyte & 0x60u));
+    const uint32_t size = is_o ? 4u + nob + 4u * fl : (fl ? 4u * (1u + fl) : 0u);
+    uint32_t agg;
+    const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg);
+    bad |= (tid == 0 && agg != bytes);
+    if (__syncthreads_or(bad)) {
+        if (tid == 0) {
+            if (bytes) mbar_wait(&s_bar, 0);  // never exit with a bulk copy in flight
+            if (d_status) atomicOr(d_status, ST_FORMAT);
+        }
+        return;
+    }
+    if (bytes) mbar_wait(&s_bar, 0);
+
+    // ---- ❷⁻¹ decode: sign field, outlier, bit planes (top plane first)
+    uint32_t a[L];
+#pragma unroll
+    for (int i = 0; i < L; i++) a[i] = 0;
+    uint32_t sign = 0;
+    if (size) {
+        uint32_t pos = phase + my_excl;
+        sign = ld_u32_unaligned(pbuf, pos);
+        pos += 4;
+        uint32_t outlier = 0;
+        if (is_o) {
+            outlier = ld_u32_unaligned(pbuf, pos);
+            if (nob < 4) outlier &= (1u << (8 * nob)) - 1u;
+            pos += nob;
+        }
+        for (int k = static_cast<int>(fl) - 1; k >= 0; k--) {
+            uint32_t w = ld_u32_unaligned(pbuf, pos + 4 * k);
+#pragma unroll
+            for (int i = L - 1; i >= 0; i--) shift_bit_into(w, a[i]);
+        }
+        if (is_o) a[0] = outlier;
+    }
+    // ---- inverse Lorenzo (prefix sum) + ❶⁻¹ dequantization
+    const auto K = make_consts(s_eb, static_cast<T *>(nullptr));
+    T x[L];
+    int qv = 0;
+#pragma unroll
+    for (int i = 0; i < L; i++) {
+        const int d = ((sign >> i) & 1u) ? -static_cast<int>(a[i]) : static_cast<int>(a[i]);
+        qv += d;
+        x[i] = dequantize(qv, K.s);
+    }
+    const bool full = b < g.nfull;
+    if (full) {
+        store_block(ostage, tid, x);
+    } else if (active) {  // ragged tail block: only valid values
+        const uint32_t valid = static_cast<uint32_t>(g.n - b * L);
+#pragma unroll
+        for (int i = 0; i < L; i++)
+            if (i < (int)valid) out[b * L + i] = x[i];
+    }
+    fence_proxy_async_smem();
+    __syncthreads();
+    const uint64_t b0 = t * BPT;
+    if (tid == 0 && b0 < g.nfull) {
+        if (Traits<T>::ROWS == 1) {
+            tma_store_2d(&tmap, 0, static_cast<int>(b0), ostage);
+        } else {
+            tma_store_2d(&tmap, 0, static_cast<int>(2 * b0), ostage);
+            if (b0 + BPT / 2 < g.nfull)
+                tma_store_2d(&tmap, 0, static_cast<int>(2 * b0 + BPT), ostage + BPT * 128);
+        }
+        bulk_commit();
+        bulk_wait0();
+    }
+}
+
+// ------------------------------------------------------------------ container index
+__global__ void container_index_kernel(const uint64_t *__restrict__ sizes, int nparts,
+                                       uint64_t *__restrict__ offsets) {
+    if (threadIdx.x == 0 && blockIdx.x == 0) {
+        uint64_t s = 0;
+        for (int r = 0; r < nparts; r++) {
+            offsets[r] = s;
+            s += sizes[r];
+        }
+        offsets[nparts] = s;
+    }
+}
+
+}  // namespace cszp2

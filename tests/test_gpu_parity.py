@@ -1,0 +1,259 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bar (BASELINE.json north_star): the compressed stream is byte-identical to the
+oracle's (whole stream, d_out pre-poisoned with 0xAA), the decompressed values
+bit-identical. At full config sizes, sampled tiles are compared byte for byte
+and properties that hold at any size (error bound, header, REL range) are
+checked on every element.
+"""
+import math
+
+import numpy as np
+import pytest
+import torch
+
+from tests import streamparse as sp
+
+pytestmark = pytest.mark.gpu
+
+cuda = pytest.importorskip("torch").cuda
+if not cuda.is_available():  # pragma: no cover
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+import oracle  # noqa: E402
+import paper_conf_sc_huangdlc24_b200 as cz  # noqa: E402
+from synthetic import CONFIGS, make_field  # noqa: E402
+
+DEV = torch.device("cuda:0")
+ENC = {"plain": oracle.PLAIN, "outlier": oracle.OUTLIER}
+EBM = {"abs": oracle.ABS, "rel": oracle.REL}
+
+
+def gpu_compress(x: torch.Tensor, eb, eb_mode, enc):
+    out = torch.full((cz.compress_bound(x.numel(), x.dtype),), 0xAA, dtype=torch.uint8, device=DEV)
+    nb = torch.zeros(1, dtype=torch.int64, device=DEV)
+    cz.compress(x, eb, eb_mode, enc, out=out, out_bytes=nb)
+    torch.cuda.synchronize()
+    total = int(nb.item())
+    return out, total
+
+
+def check_roundtrip(xh: np.ndarray, eb, eb_mode, enc, compare_stream=True):
+    x = torch.from_numpy(xh).to(DEV)
+    out, total = gpu_compress(x, eb, eb_mode, enc)
+    ref, rc = oracle.compress(xh, eb, EBM[eb_mode], ENC[enc])
+    got = out[:total].cpu().numpy()
+    h = sp.header(got)
+    assert total == ref.size == h["total_bytes"]
+    if rc == oracle.ERR_RANGE:
+        assert h["status"] == 3
+        np.testing.assert_array_equal(got[:64], ref[:64])  # parity covers the header only
+        st = torch.zeros(1, dtype=torch.int32, device=DEV)
+        cz.decompress(out, xh.size, x.dtype, status=st)
+        torch.cuda.synchronize()
+        assert int(st.item()) == 3
+        return None
+    assert rc == oracle.OK
+    if compare_stream:
+        if not np.array_equal(got, ref):
+            bad = np.nonzero(got != ref)[0]
+            raise AssertionError(f"stream differs at {bad.size} bytes, first {bad[:8]} (total {total})")
+    st = torch.zeros(1, dtype=torch.int32, device=DEV)
+    y = torch.full_like(x, float("nan"))
+    cz.decompress(out, xh.size, x.dtype, out=y, status=st)
+    torch.cuda.synchronize()
+    assert int(st.item()) == 0
+    yr, rc = oracle.decompress(ref, xh.size, xh.dtype)
+    assert rc == oracle.OK
+    iv = np.uint32 if xh.dtype == np.float32 else np.uint64
+    np.testing.assert_array_equal(y.cpu().numpy().view(iv), yr.view(iv))
+    return got
+
+
+SIZES = [0, 1, 31, 32, 33, 1000, 8192, 8192 * 3 + 32 * 5 + 11, 100003]
+
+
+@pytest.mark.parametrize("n", SIZES)
+@pytest.mark.parametrize("enc", ["plain", "outlier"])
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_small_sizes_rel(n, enc, dtype):
+    rng = np.random.default_rng(n + 17)
+    xh = (np.cumsum(rng.standard_normal(n)) * 0.3 + 10).astype(dtype)
+    check_roundtrip(xh, 1e-3, "rel", enc)
+
+
+@pytest.mark.parametrize("eb", [0.5, 1e-1, 1e-3, 1e-6])
+@pytest.mark.parametrize("enc", ["plain", "outlier"])
+def test_abs_bounds_noise(eb, enc):
+    """Random noise: every fixed length up to ~24 bits appears."""
+    rng = np.random.default_rng(int(1 / eb))
+    xh = (rng.standard_normal(40000) * rng.choice([1e-3, 1.0, 100.0], 40000)).astype(np.float32)
+    check_roundtrip(xh, eb, "abs", enc)
+
+
+def test_ties_round_half_even():
+    xh = (np.arange(-5000, 5000) + 0.5).astype(np.float32)
+    got = check_roundtrip(xh, 0.5, "abs", "plain")
+    np.testing.assert_array_equal(sp.parse(got)["q"], np.rint(xh).astype(np.int64))
+
+
+@pytest.mark.parametrize("enc", ["plain", "outlier"])
+def test_special_fields(enc):
+    n = 8192 * 2 + 77
+    check_roundtrip(np.zeros(n, np.float32), 1e-4, "abs", enc)            # zero blocks
+    check_roundtrip(np.full(n, 5.0, np.float32), 0.5, "abs", enc)         # constant
+    check_roundtrip(np.full(n, -3.25, np.float64), 1e-2, "rel", enc)      # zero range
+    alt = np.where(np.arange(n) % 2 == 0, 1073741760.0, -1073741760.0).astype(np.float32)
+    check_roundtrip(alt, 0.5, "abs", enc)                                 # fl = 31 everywhere
+    xh = np.zeros(n, np.float32)
+    xh[::97] = 1000.0                                                     # sparse spikes
+    check_roundtrip(xh, 1e-3, "abs", enc)
+
+
+def test_range_status_header_parity():
+    xh = np.linspace(0, 1, 10000).astype(np.float32)
+    xh[5000] = 3e9
+    check_roundtrip(xh, 0.5, "abs", "outlier")
+    xh[5000] = np.nan
+    check_roundtrip(xh, 0.5, "abs", "plain")
+    xh = np.array([1.0, np.inf, 2.0] * 100, np.float32)
+    check_roundtrip(xh, 1e-3, "rel", "plain")  # infinite range -> RANGE
+
+
+@pytest.mark.parametrize("cfg", ["cfg1", "cfg2"])
+@pytest.mark.parametrize("enc", ["plain", "outlier"])
+def test_configs_small_full_stream(cfg, enc):
+    """BASELINE configs 1 and 2 at full size: whole-stream byte parity."""
+    spec = CONFIGS[cfg]
+    xh = make_field(cfg, DEV).cpu().numpy()
+    for eb in spec.ebs:
+        check_roundtrip(xh, eb, spec.eb_mode, enc)
+
+
+def test_decompress_rejects_corrupt_streams():
+    rng = np.random.default_rng(0)
+    x = torch.from_numpy(np.cumsum(rng.standard_normal(50000)).astype(np.float32)).to(DEV)
+    out, total = gpu_compress(x, 1e-2, "abs", "outlier")
+
+    def status(buf, n=x.numel(), dtype=torch.float32):
+        st = torch.zeros(1, dtype=torch.int32, device=DEV)
+        cz.decompress(buf, n, dtype, status=st)
+        torch.cuda.synchronize()
+        return int(st.item())
+
+    assert status(out) == 0
+    bad = out.clone(); bad[0] ^= 1
+    assert status(bad) == 4
+    assert status(out, x.numel() + 1) == 4
+    assert status(out, x.numel(), torch.float64) == 4
+    nb, T, O, D = sp.geometry(x.numel())
+    bad = out.clone(); bad[O + 3] = 0x60  # reserved bits
+    assert status(bad) == 4
+    bad = out.clone(); bad[64 + 8 * 2 + 7] = 0  # index flag cleared
+    assert status(bad) == 4
+
+
+def test_container_index():
+    sizes = torch.tensor([100, 0, 37, 5], dtype=torch.int64, device=DEV)
+    off = cz.container_index(sizes)
+    assert off.cpu().tolist() == [0, 100, 100, 137, 142]
+
+
+def test_host_buffer_api():
+    rng = np.random.default_rng(9)
+    xh = np.cumsum(rng.standard_normal(70001)).astype(np.float32)
+    h_in = torch.from_numpy(xh).pin_memory()
+    d_in = torch.empty(xh.size, dtype=torch.float32, device=DEV)
+    d_out = torch.empty(cz.compress_bound(xh.size), dtype=torch.uint8, device=DEV)
+    h_out = torch.empty(cz.compress_bound(xh.size), dtype=torch.uint8).pin_memory()
+    nbytes = cz.compress_host(h_in, 1e-3, "rel", "outlier", d_in, d_out, h_out)
+    ref, _ = oracle.compress(xh, 1e-3, oracle.REL, oracle.OUTLIER)
+    np.testing.assert_array_equal(h_out[:nbytes].numpy(), ref)
+    h_y = torch.empty(xh.size, dtype=torch.float32).pin_memory()
+    st = torch.zeros(1, dtype=torch.int32, device=DEV)
+    cz.decompress_host(h_out, nbytes, d_out, d_in, h_y, status=st)
+    yr, _ = oracle.decompress(ref, xh.size)
+    np.testing.assert_array_equal(h_y.numpy().view(np.uint32), yr.view(np.uint32))
+
+
+# ---------------------------------------------------------------- full-size configs
+
+def _sampled_tile_parity(x: torch.Tensor, out: torch.Tensor, y: torch.Tensor, enc: str, tiles):
+    """Compare sampled tiles of a full-size GPU stream with the oracle run on
+    exactly those blocks (block encoding is position independent; FORMAT.md §2)."""
+    n = x.numel()
+    h = cz.read_header(out)
+    nb, T, O, D = sp.geometry(n)
+    index = out[64:64 + 8 * T].cpu().numpy().view("<u8")
+    assert np.all(index >> np.uint64(62) == 2)
+    incl = index & np.uint64((1 << 62) - 1)
+    assert int(incl[-1]) == h["payload_bytes"]
+    for t in tiles:
+        b0, b1 = t * 256, min(nb, (t + 1) * 256)
+        v0, v1 = b0 * 32, min(n, b1 * 32)
+        xs = x[v0:v1].cpu().numpy()
+        ref, rc = oracle.compress(xs, h["eb_abs"], oracle.ABS, ENC[enc])
+        assert rc == oracle.OK
+        rp = sp.parse(ref)
+        _, _, rO, rD = rp["geometry"]
+        e0 = 0 if t == 0 else int(incl[t - 1])
+        e1 = int(incl[t])
+        np.testing.assert_array_equal(out[O + b0:O + b1].cpu().numpy(), ref[rO:rO + (b1 - b0)])
+        np.testing.assert_array_equal(out[D + e0:D + e1].cpu().numpy(), ref[rD:rD + (e1 - e0)])
+        yr, rc = oracle.decompress(ref, xs.size, xs.dtype)
+        iv = np.uint32 if xs.dtype == np.float32 else np.uint64
+        np.testing.assert_array_equal(y[v0:v1].cpu().numpy().view(iv), yr.view(iv))
+
+
+def _error_bound_all(x, y, eb_abs):
+    xd, yd = x.double(), y.double()
+    err = (xd - yd).abs()
+    mag = torch.maximum(xd.abs(), yd.abs())
+    if x.dtype == torch.float32:
+        bound = eb_abs * (1 + 2.0 ** -20) + 2.0 ** -21 * mag
+    else:
+        bound = eb_abs * (1 + 2.0 ** -40) + 2.0 ** -50 * mag
+    assert bool((err <= bound).all())
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("cfg", ["cfg3a", "cfg3b", "cfg4a", "cfg4b"])
+def test_full_size_configs(cfg):
+    spec = CONFIGS[cfg]
+    x = make_field(cfg, DEV)
+    n = x.numel()
+    nb, T, O, D = sp.geometry(n)
+    lam = spec.ebs[-1]
+    r = float(x.max().double() - x.min().double())
+    for enc in spec.modes:
+        out, total = gpu_compress(x, lam, spec.eb_mode, enc)
+        h = cz.read_header(out)
+        assert h["status"] == 0 and h["total_bytes"] == total
+        assert h["eb_abs"] == lam * r  # REL range from torch's own min/max
+        rng = np.random.default_rng(T)
+        tiles = sorted(set([0, T - 1, T // 2] + list(rng.integers(0, T, 6))))
+        y = cz.decompress(out, n, x.dtype)
+        _sampled_tile_parity(x, out, y, enc, tiles)
+        _error_bound_all(x, y, h["eb_abs"])
+        del y, out
+        torch.cuda.empty_cache()
+
+
+@pytest.mark.slow
+def test_config5_single_gpu_sampled():
+    """2048^3 f32 (32 GiB) on one B200: sampled-tile byte parity + bound on every element."""
+    free, _ = torch.cuda.mem_get_info()
+    if free < 110 * 2**30:
+        pytest.skip("needs ~110 GiB free device memory")
+    spec = CONFIGS["cfg5"]
+    x = make_field("cfg5", DEV)
+    n = x.numel()
+    nb, T, O, D = sp.geometry(n)
+    out, total = gpu_compress(x, 1e-4, "rel", "outlier")
+    h = cz.read_header(out)
+    assert h["status"] == 0 and h["eb_abs"] == 1e-4 * float(x.max().double() - x.min().double())
+    rng = np.random.default_rng(5)
+    y = cz.decompress(out, n, x.dtype)
+    _sampled_tile_parity(x, out, y, "outlier", sorted(set([0, T - 1] + list(rng.integers(0, T, 4)))))
+    for s in range(0, n, 1 << 30):
+        _error_bound_all(x[s:s + (1 << 30)], y[s:s + (1 << 30)], h["eb_abs"])
