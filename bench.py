@@ -1,0 +1,467 @@
+#!/usr/bin/env python
+"""Benchmark of the cuSZp2 hot path on B200 (BASELINE.json metric).
+
+Workload (default): BASELINE config 5 — the 2048^3 f32 NYX-shaped synthetic
+field (32 GiB), REL 1e-4, Outlier-FLE, slab-sharded across the ranks (strong
+scaling: the field is fixed, each of N ranks owns 2^33/N values). One step =
+one pass of the whole hot path: REL resolve (memset + device min/max) →
+fused compression kernel → [N>1: NCCL all-gather of the per-rank compressed
+sizes + container index kernel] → fused decompression kernel.
+
+value = round-trip throughput: uncompressed bytes of the whole field ÷ (max
+over ranks of the device time of compress + decompress), GB/s. comp_gbs and
+decomp_gbs give the two directions separately (same clock).
+
+Launch: python bench.py [--gpus N --steps K --warmup W] (torchrun for N>1);
+        python bench.py --impl reference  → the CPU oracle on host cores.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from synthetic import CONFIGS, make_field  # noqa: E402
+
+METRIC = "comp/decomp end-to-end GB/s per B200 & at 2/4/8 GPUs; CR and PSNR at REL 1e-4"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="cfg5")
+    ap.add_argument("--enc", default="outlier", choices=["plain", "outlier"])
+    ap.add_argument("--eb", type=float, default=None)
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--e2e-max-gib", type=float, default=40.0,
+                    help="cap on the per-rank slab used for the host-buffer e2e leg")
+    ap.add_argument("--cpu-sample-log2", type=int, default=28,
+                    help="values in the oracle cpu_baseline sample (2^k)")
+    ap.add_argument("--no-plain", action="store_true", help="skip the secondary Plain-mode pass")
+    return ap.parse_args()
+
+
+# ----------------------------------------------------------------- helpers
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def slab(n: int, world: int, rank: int):
+    """Block-aligned contiguous slab of rank r."""
+    S = -(-n // world)
+    S = -(-S // 32) * 32
+    s0 = min(n, rank * S)
+    return s0, min(n, s0 + S) - s0
+
+
+def load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.15)
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for l in self.lines:
+            f = [x.strip() for x in l.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = float(f[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def traffic_from_profiles(kernel_key: str):
+    """dram read+write bytes per launch from the committed ncu --set full summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_full_summary.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d.get(kernel_key, {}).get("dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+# ----------------------------------------------------------------- reference arm (CPU oracle)
+
+def run_reference(args):
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return 0
+    import oracle
+
+    spec = CONFIGS[args.config]
+    lam = args.eb if args.eb is not None else spec.ebs[-1]
+    enc = oracle.OUTLIER if args.enc == "outlier" else oracle.PLAIN
+    ebm = oracle.REL if spec.eb_mode == "rel" else oracle.ABS
+    torch.set_num_threads(os.cpu_count() or 1)
+    sample = 1 << 24
+    x = make_field(args.config, "cpu", 0, sample).numpy()
+    w = x.itemsize
+    for _ in range(args.warmup):
+        s, _ = oracle.compress(x, lam, ebm, enc)
+        oracle.decompress(s, x.size, x.dtype)
+    tc = td = 0.0
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        s, rc = oracle.compress(x, lam, ebm, enc)
+        t1 = time.perf_counter()
+        y, rc2 = oracle.decompress(s, x.size, x.dtype)
+        t2 = time.perf_counter()
+        tc += t1 - t0
+        td += t2 - t1
+    gb = x.nbytes * args.steps / 1e9
+    value = gb / (tc + td)
+    desc = (f"first 2^24 values ({x.nbytes/2**20:.0f} MiB) of the {spec.name} field per step, "
+            f"single-threaded C oracle, REL {lam:g} {args.enc}")
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GB/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round((tc + td) / args.steps * 1e3, 3), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f32" if w == 4 else "f64",
+        "data": "synthetic",
+        "config": {"workload": f"{args.config} {spec.name} REL {lam:g} {args.enc} (oracle sample)",
+                   "sample_values": sample},
+        "comp_gbs": round(gb / tc, 4), "decomp_gbs": round(gb / td, 4),
+        "cr": round(x.nbytes / s.size, 3),
+        "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                         "sample": desc},
+        "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ----------------------------------------------------------------- our arm
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import paper_conf_sc_huangdlc24_b200 as cz
+
+    rank, world, local = dist_env()
+    if world != args.gpus and world > 1:
+        print(f"warning: WORLD_SIZE={world} != --gpus {args.gpus}", file=sys.stderr)
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+
+        dist.init_process_group("nccl", device_id=dev)
+
+    spec = CONFIGS[args.config]
+    lam = args.eb if args.eb is not None else spec.ebs[-1]
+    n_total = spec.n
+    s0, cnt = slab(n_total, world, rank)
+    w = spec.itemsize
+    dtype = spec.dtype
+
+    x = make_field(args.config, dev, start=s0, count=cnt)
+    bound = cz.compress_bound(cnt, dtype)
+    out = torch.empty(bound, dtype=torch.uint8, device=dev)
+    nbytes = torch.zeros(1, dtype=torch.int64, device=dev)
+    y = torch.empty_like(x)
+    sizes = torch.zeros(world, dtype=torch.int64, device=dev)
+    offsets = torch.zeros(world + 1, dtype=torch.int64, device=dev)
+    stream = torch.cuda.current_stream(dev)
+
+    def step(evs=None, enc=args.enc):
+        if evs:
+            evs[0].record(stream)
+        cz.compress_prepare(x, lam, spec.eb_mode, out, stream=stream)
+        if evs:
+            evs[1].record(stream)
+        cz.compress_encode(x, lam, spec.eb_mode, enc, out, nbytes, stream=stream)
+        if evs:
+            evs[2].record(stream)
+        if world > 1:
+            dist.all_gather_into_tensor(sizes, nbytes)
+            cz.container_index(sizes, out=offsets, stream=stream)
+        if evs:
+            evs[3].record(stream)
+        cz.decompress(out, cnt, dtype, out=y, stream=stream)
+        if evs:
+            evs[4].record(stream)
+
+    for _ in range(max(3, args.warmup)):
+        step()
+    torch.cuda.synchronize()
+
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(5)] for _ in range(args.steps)]
+    t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    if dist:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        t_start.record(stream)
+        for k in range(args.steps):
+            step(evs[k])
+        t_end.record(stream)
+        torch.cuda.synchronize()
+    if dist:
+        dist.barrier()
+    total_ms = t_start.elapsed_time(t_end)
+    ph = np.array([[e[i].elapsed_time(e[i + 1]) for i in range(4)] for e in evs])  # ms
+    prep_ms, enc_ms, gather_ms, dec_ms = ph.mean(axis=0)
+    comp_ms = prep_ms + enc_ms + gather_ms
+    stream_bytes = int(nbytes.item())
+
+    # max over ranks of every timing (device clocks), sum of stream bytes
+    vec = torch.tensor([total_ms, comp_ms, dec_ms, prep_ms, enc_ms, gather_ms], dtype=torch.float64, device=dev)
+    sb = torch.tensor([stream_bytes], dtype=torch.int64, device=dev)
+    if dist:
+        dist.all_reduce(vec, op=dist.ReduceOp.MAX)
+        dist.all_reduce(sb, op=dist.ReduceOp.SUM)
+    total_ms, comp_ms, dec_ms, prep_ms, enc_ms, gather_ms = vec.tolist()
+    stream_total = int(sb.item())
+
+    # CR + PSNR of the whole field (after the timed region; PSNR per reading R-16)
+    hdr = cz.read_header(out)
+    mse_sum = torch.zeros(1, dtype=torch.float64, device=dev)
+    mn = torch.full((1,), float("inf"), dtype=torch.float64, device=dev)
+    mx = torch.full((1,), -float("inf"), dtype=torch.float64, device=dev)
+    for c0 in range(0, cnt, 1 << 28):
+        xs, ys = x[c0:c0 + (1 << 28)].double(), y[c0:c0 + (1 << 28)].double()
+        mse_sum += ((xs - ys) ** 2).sum()
+        mn = torch.minimum(mn, xs.min().view(1))
+        mx = torch.maximum(mx, xs.max().view(1))
+        del xs, ys
+    if dist:
+        dist.all_reduce(mse_sum)
+        dist.all_reduce(mn, op=dist.ReduceOp.MIN)
+        dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+    mse = float(mse_sum.item()) / n_total
+    rng_v = float(mx.item() - mn.item())
+    psnr = 20 * math.log10(rng_v) - 10 * math.log10(mse) if mse > 0 else float("inf")
+
+    gb_field = n_total * w / 1e9
+    value = gb_field / ((comp_ms + dec_ms) * 1e-3)
+    comp_gbs = gb_field / (comp_ms * 1e-3)
+    decomp_gbs = gb_field / (dec_ms * 1e-3)
+
+    # roofline of the dominant kernel (per rank, algorithmic bytes / avg duration)
+    peak, peak_src = load_peaks()
+    slab_bytes = cnt * w
+    enc_bytes = slab_bytes + stream_bytes           # read field, write stream
+    dec_bytes = stream_bytes + slab_bytes           # read stream, write field
+    kern = {
+        "compress_kernel": {"ms": enc_ms, "bytes": enc_bytes},
+        "decompress_kernel": {"ms": dec_ms, "bytes": dec_bytes},
+        "minmax_kernel": {"ms": prep_ms, "bytes": slab_bytes},
+    }
+    for k, v in kern.items():
+        v["gbs"] = v["bytes"] / (v["ms"] * 1e-3) / 1e9
+        v["frac"] = v["gbs"] / peak
+    dom = max(("compress_kernel", "decompress_kernel"), key=lambda k: kern[k]["ms"])
+    roof = {"bound": "hbm", "kernel": dom, "achieved": round(kern[dom]["gbs"], 1), "peak": peak,
+            "unit": "GB/s", "frac": round(kern[dom]["frac"], 4),
+            "traffic": traffic_from_profiles(dom), "peak_source": peak_src,
+            "algorithmic_bytes_per_launch": kern[dom]["bytes"],
+            "kernels": {k: {"ms": round(v["ms"], 4), "gbs": round(v["gbs"], 1), "frac": round(v["frac"], 4)}
+                        for k, v in kern.items()}}
+    clocks = clk.summary()
+
+    # secondary: Plain mode (both encoding modes are part of config 5)
+    plain = None
+    if not args.no_plain and args.enc != "plain":
+        for _ in range(2):
+            step(enc="plain")
+        pe = [[torch.cuda.Event(enable_timing=True) for _ in range(5)] for _ in range(3)]
+        for k in range(3):
+            step(pe[k], enc="plain")
+        torch.cuda.synchronize()
+        pp = np.array([[e[i].elapsed_time(e[i + 1]) for i in range(4)] for e in pe]).mean(axis=0)
+        pv = torch.tensor([pp[0] + pp[1] + pp[2], pp[3]], dtype=torch.float64, device=dev)
+        pbytes = torch.tensor([int(nbytes.item())], dtype=torch.int64, device=dev)
+        if dist:
+            dist.all_reduce(pv, op=dist.ReduceOp.MAX)
+            dist.all_reduce(pbytes)
+        plain = {"comp_gbs": round(gb_field / (pv[0].item() * 1e-3), 1),
+                 "decomp_gbs": round(gb_field / (pv[1].item() * 1e-3), 1),
+                 "cr": round(n_total * w / int(pbytes.item()), 3)}
+        step()  # leave the main-mode stream in `out`
+        torch.cuda.synchronize()
+
+    # cpu_baseline: the oracle as it stands, on a bounded sample, rank 0 at N=1 only
+    cpu = None
+    if rank == 0 and world == 1:
+        cpu = run_cpu_baseline(args, x, lam, spec)
+
+    # e2e through the host-buffer C-ABI calls (pinned host memory, copies timed)
+    e2e = run_e2e(args, cz, x, y, out, dev, stream, lam, spec, dist, world, n_total, w)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
+            "steps": args.steps, "warmup": max(3, args.warmup),
+            "ms_per_step": round(total_ms / args.steps, 4), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None,
+            "dtype": "f32" if w == 4 else "f64", "data": "synthetic",
+            "config": {"workload": f"{args.config}: {spec.name} {spec.dtype} field, REL {lam:g}, "
+                                   f"{args.enc}-FLE, slab-sharded over {world} rank(s)",
+                       "n_values": n_total, "values_per_rank": cnt, "eb_mode": spec.eb_mode,
+                       "eb": lam, "enc_mode": args.enc,
+                       "l2": "inputs larger than L2 (field >> 126 MB); no flush needed",
+                       "parallelism": f"slab x{world}, NCCL all-gather of compressed sizes"},
+            "comp_gbs": round(comp_gbs, 1), "decomp_gbs": round(decomp_gbs, 1),
+            "cr": round(n_total * w / stream_total, 3), "psnr_db": round(psnr, 3),
+            "eb_abs_rank0": hdr["eb_abs"],
+            "phase_ms": {"prepare_minmax": round(prep_ms, 4), "compress_kernel": round(enc_ms, 4),
+                         "allgather_index": round(gather_ms, 4), "decompress_kernel": round(dec_ms, 4)},
+            "roofline": roof,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "clocks": clocks,
+            "gpu_launches": args.steps * (3 + (1 if world > 1 else 0)),
+            "plain_mode": plain,
+        }
+        print(json.dumps(line), flush=True)
+    if dist:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def run_e2e(args, cz, x, y, out, dev, stream, lam, spec, dist, world, n_total, w):
+    """Same metric through cszp2_compress_host / cszp2_decompress_host: every
+    step copies its input from pinned host memory and its result back. Reuses
+    the device buffers of the main run (x's contents are consumed)."""
+    cap = int(args.e2e_max_gib * 2**30 // w) // 32 * 32
+    m = min(x.numel(), cap)
+    h_in = torch.empty(m, dtype=x.dtype, pin_memory=True)
+    h_in.copy_(x[:m])
+    d_in, d_out, d_y = y[:m], out, x[:m]  # work buffers (caller-owned, FORMAT.md-sized)
+    h_out = torch.empty(cz.compress_bound(m, x.dtype), dtype=torch.uint8, pin_memory=True)
+    h_y = torch.empty(m, dtype=x.dtype, pin_memory=True)
+    st = torch.zeros(1, dtype=torch.int32, device=dev)
+    nbytes = cz.compress_host(h_in, lam, spec.eb_mode, args.enc, d_in, d_out, h_out, stream)  # warm-up
+    cz.decompress_host(h_out, nbytes, d_out, d_y, h_y, status=st, stream=stream)
+    tc = td = 0.0
+    for _ in range(args.e2e_steps):
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0, e1, e2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+        e0.record(stream)
+        nbytes = cz.compress_host(h_in, lam, spec.eb_mode, args.enc, d_in, d_out, h_out, stream)
+        e1.record(stream)
+        cz.decompress_host(h_out, nbytes, d_out, d_y, h_y, status=st, stream=stream)
+        e2.record(stream)
+        torch.cuda.synchronize()
+        tc += e0.elapsed_time(e1)
+        td += e1.elapsed_time(e2)
+    v = torch.tensor([tc / args.e2e_steps, td / args.e2e_steps], dtype=torch.float64, device=dev)
+    mm = torch.tensor([m], dtype=torch.int64, device=dev)
+    if dist:
+        dist.all_reduce(v, op=dist.ReduceOp.MAX)
+        dist.all_reduce(mm)
+    tcm, tdm = v.tolist()
+    gb = int(mm.item()) * w / 1e9
+    # sanity: the host result honours the bound on a prefix (full parity is in tests/)
+    k = min(m, 1 << 22)
+    eb_abs = cz.read_header(d_out, stream)["eb_abs"]
+    a, b = h_in[:k].double(), h_y[:k].double()
+    okb = bool(((a - b).abs() <= eb_abs * (1 + 2.0 ** -20) + 2.0 ** -21 * torch.maximum(a.abs(), b.abs())).all())
+    res = {"value": round(gb / ((tcm + tdm) * 1e-3), 2), "unit": "GB/s",
+           "comp_gbs": round(gb / (tcm * 1e-3), 2), "decomp_gbs": round(gb / (tdm * 1e-3), 2),
+           "h2d_bytes_per_step": m * w + nbytes, "d2h_bytes_per_step": nbytes + m * w,
+           "values_per_rank": m, "status_ok": int(st.item()) == 0, "bound_ok_prefix": okb,
+           "api": "cszp2_compress_host + cszp2_decompress_host (pinned host buffers)"}
+    if m < x.numel():
+        res["sample"] = f"first {m} values of each rank's slab (--e2e-max-gib {args.e2e_max_gib})"
+    del h_in, h_out, h_y
+    return res
+
+
+def run_cpu_baseline(args, x, lam, spec):
+    import oracle
+
+    m = min(x.numel(), 1 << args.cpu_sample_log2)
+    xs = x[:m].cpu().numpy()
+    ebm = oracle.REL if spec.eb_mode == "rel" else oracle.ABS
+    enc = oracle.OUTLIER if args.enc == "outlier" else oracle.PLAIN
+    t0 = time.perf_counter()
+    s, rc = oracle.compress(xs, lam, ebm, enc)
+    t1 = time.perf_counter()
+    yh, rc2 = oracle.decompress(s, m, xs.dtype)
+    t2 = time.perf_counter()
+    gb = xs.nbytes / 1e9
+    return {"value": round(gb / (t2 - t0), 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+            "comp_gbs": round(gb / (t1 - t0), 4), "decomp_gbs": round(gb / (t2 - t1), 4),
+            "seconds": round(t2 - t0, 2),
+            "sample": f"first {m} values ({xs.nbytes / 2**30:.2f} GiB) of the rank-0 slab, one "
+                      f"compress + decompress, single-threaded C oracle (REL range of the sample)"}
+
+
+if __name__ == "__main__":
+    sys.exit(main())
