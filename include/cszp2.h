@@ -61,8 +61,9 @@ typedef struct {
     uint64_t total_bytes;
 } cszp2_header;
 
-/* Bytes a compressed stream of n values may occupy (FORMAT.md §2); d_out of
- * cszp2_compress must hold this many bytes. Returns 0 for an invalid dtype. */
+/* Bytes d_out of cszp2_compress must hold: the largest stream of n values
+ * (FORMAT.md §2, roundup16(D + 128*nb)) plus 16 bytes of scratch used by the
+ * kernel's tile ticket. Returns 0 for an invalid dtype. */
 uint64_t cszp2_compress_bound(uint64_t n, int dtype);
 
 /* Compression (P:84-102 problem statement; Fig 4 workflow ❶-❹).

@@ -76,6 +76,34 @@ int set_smem(K kernel, int bytes) {
 
 int launch_status() { return cudaGetLastError() == cudaSuccess ? CSZP2_OK : CSZP2_ERR_CUDA; }
 
+// stream bound without the 16-byte scratch tail (FORMAT.md §2)
+uint64_t stream_bound(const Geom &g) { return roundup16(g.D + static_cast<uint64_t>(4 * L) * g.nb); }
+
+int sm_count() {
+    static int sms = 0;
+    if (!sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (sms <= 0) sms = 148;
+    }
+    return sms;
+}
+
+// persistent grid: every CTA resident (occupancy x SMs), never more than tiles
+template <typename K>
+unsigned persistent_grid(K kernel, int smem, uint64_t tiles, int *cache) {
+    if (*cache <= 0) {
+        int per_sm = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, NT, smem) != cudaSuccess ||
+            per_sm < 1)
+            per_sm = 1;
+        *cache = per_sm * sm_count();
+    }
+    const uint64_t t = tiles ? tiles : 1;
+    return static_cast<unsigned>(t < static_cast<uint64_t>(*cache) ? t : *cache);
+}
+
 int check_compress_args(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
                         const void *d_out) {
     if (!wsize(dtype) || !d_out || (!d_in && n)) return CSZP2_ERR_ARG;
@@ -88,9 +116,7 @@ int check_compress_args(const void *d_in, uint64_t n, int dtype, double eb, int 
 
 template <typename T>
 int launch_minmax(const void *d_in, uint64_t n, double lambda, void *d_out, cudaStream_t st) {
-    int dev = 0, sms = 148;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int sms = sm_count();
     const uint64_t nvec = n / (16 / sizeof(T));
     uint64_t want = (nvec + 255) / 256;
     int grid = static_cast<int>(want < 1 ? 1 : (want > (uint64_t)sms * 8 ? (uint64_t)sms * 8 : want));
@@ -104,9 +130,12 @@ int launch_compress(const void *d_in, const Geom &g, double eb, int eb_mode, int
                     void *d_out, uint64_t *d_out_bytes, cudaStream_t st) {
     static std::once_flag once;
     static int attr_rc = CSZP2_OK;
+    static int grid_cache = 0;
     constexpr int smem = compress_smem_bytes<T>();
     std::call_once(once, [] { attr_rc = set_smem(compress_kernel<T, OUTLIER>, smem); });
     if (attr_rc) return attr_rc;
+    const unsigned grid = persistent_grid(compress_kernel<T, OUTLIER>, smem, g.T, &grid_cache);
+    unsigned *ticket = reinterpret_cast<unsigned *>(static_cast<uint8_t *>(d_out) + stream_bound(g));
     CUtensorMap map;
     int rc = make_tmap(&map, d_in, Traits<T>::DTYPE, g.nfull);
     if (rc) return rc;
@@ -115,10 +144,9 @@ int launch_compress(const void *d_in, const Geom &g, double eb, int eb_mode, int
                (static_cast<uint32_t>(enc_mode) << 16) | (5u << 24);
     hs.eb_mode = static_cast<uint32_t>(eb_mode);
     hs.eb_user = eb;
-    const uint64_t grid = g.T ? g.T : 1;
-    compress_kernel<T, OUTLIER><<<static_cast<unsigned>(grid), NT, smem, st>>>(
+    compress_kernel<T, OUTLIER><<<grid, NT, smem, st>>>(
         map, static_cast<const T *>(d_in), g, eb, eb_mode == CSZP2_EB_REL ? 1 : 0,
-        static_cast<uint8_t *>(d_out), d_out_bytes, hs);
+        static_cast<uint8_t *>(d_out), ticket, d_out_bytes, hs);
     return launch_status();
 }
 
@@ -127,14 +155,15 @@ int launch_decompress(const void *d_cmp, void *d_out, const Geom &g, int *d_stat
                       cudaStream_t st) {
     static std::once_flag once;
     static int attr_rc = CSZP2_OK;
+    static int grid_cache = 0;
     constexpr int smem = decompress_smem_bytes<T>();
     std::call_once(once, [] { attr_rc = set_smem(decompress_kernel<T>, smem); });
     if (attr_rc) return attr_rc;
+    const unsigned grid = persistent_grid(decompress_kernel<T>, smem, g.T, &grid_cache);
     CUtensorMap map;
     int rc = make_tmap(&map, d_out, Traits<T>::DTYPE, g.nfull);
     if (rc) return rc;
-    const uint64_t grid = g.T ? g.T : 1;
-    decompress_kernel<T><<<static_cast<unsigned>(grid), NT, smem, st>>>(
+    decompress_kernel<T><<<grid, NT, smem, st>>>(
         map, static_cast<const uint8_t *>(d_cmp), static_cast<T *>(d_out), g, d_status);
     return launch_status();
 }
@@ -147,8 +176,8 @@ const char *cszp2_version(void) { return "cszp2 1.0 sm_100a"; }
 
 uint64_t cszp2_compress_bound(uint64_t n, int dtype) {
     if (!wsize(dtype)) return 0;
-    Geom g = geometry(n);
-    return roundup16(g.D + static_cast<uint64_t>(4 * L) * g.nb);
+    // the stream's worst case plus 16 bytes of scratch (the compression ticket)
+    return stream_bound(geometry(n)) + 16;
 }
 
 int cszp2_compress_prepare(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
@@ -156,7 +185,9 @@ int cszp2_compress_prepare(const void *d_in, uint64_t n, int dtype, double eb, i
     int rc = check_compress_args(d_in, n, dtype, eb, eb_mode, d_out);
     if (rc) return rc;
     Geom g = geometry(n);
-    if (cudaMemsetAsync(d_out, 0, g.O, S(stream)) != cudaSuccess) return CSZP2_ERR_CUDA;
+    if (cudaMemsetAsync(d_out, 0, g.O, S(stream)) != cudaSuccess ||
+        cudaMemsetAsync(static_cast<uint8_t *>(d_out) + stream_bound(g), 0, 16, S(stream)) != cudaSuccess)
+        return CSZP2_ERR_CUDA;
     if (eb_mode == CSZP2_EB_REL)
         return dtype == CSZP2_F32 ? launch_minmax<float>(d_in, n, eb, d_out, S(stream))
                                   : launch_minmax<double>(d_in, n, eb, d_out, S(stream));

@@ -24,6 +24,7 @@ namespace cszp2 {
 constexpr int L = 32;      // values per block
 constexpr int BPT = 256;   // blocks per tile (FORMAT.md §1)
 constexpr int NT = 256;    // threads per CTA: one block per thread
+constexpr int TMA_TID = 32;  // compression: the thread that claims tiles and owns the TMA traffic
 constexpr uint32_t MAGIC = 0x325A5343u;
 constexpr uint64_t FLAG_A = 1ull << 62;   // lookback: aggregate available
 constexpr uint64_t FLAG_P = 2ull << 62;   // lookback: inclusive prefix available
@@ -186,42 +187,90 @@ __device__ __forceinline__ uint32_t cta_exclusive_scan(uint32_t v, uint32_t *s_w
     return base + inc - v;
 }
 
-// ❸ Decoupled lookback (Fig 13; after Merrill & Garland [25]).
-// Executed by one full warp. Tile t publishes (A | aggregate), then walks back
-// over its predecessors' descriptors 32 at a time, summing aggregates until it
-// meets an inclusive prefix (P); then publishes (P | inclusive). The final
-// descriptors ARE the stream's tile index (FORMAT.md §2). Returns the
-// exclusive prefix of tile t.
-__device__ __forceinline__ uint64_t lookback(uint64_t *index, uint64_t t, uint64_t agg) {
+// ❸ Decoupled lookback (Fig 13; after Merrill & Garland [25]), split
+// so that no CTA ever sits on an unpublished tile while it waits:
+//   publish_aggregate: tile t announces (A | aggregate) — (P | aggregate) for
+//                      tile 0 — as soon as its blocks are encoded;
+//   lookback_issue /   one iteration later, a full warp loads its predecessors'
+//   lookback_finish:   descriptors in windows of 256 (8 per lane, nearest first;
+//                      loads issued before the next tile's encode so their latency
+//                      hides behind it), sums aggregates down to the nearest
+//                      inclusive prefix (P) and publishes (P | inclusive).
+// Descriptor: flag (bits 63-62: 0 Waiting, 1 A, 2 P) | RANGE bit 61 (A: this
+// tile saw an out-of-range value; P: some tile <= t did) | value (bits 60-0).
+// Nothing but the descriptors themselves is communicated through them, so all
+// accesses are relaxed (no membar on the critical path). The final descriptors
+// ARE the stream's tile index (FORMAT.md §2; bit 61 is 0 in every valid stream).
+constexpr int LB_PER_LANE = 8;
+constexpr uint64_t BIT_RANGE = 1ull << 61;
+constexpr uint64_t VAL61 = BIT_RANGE - 1;
+
+__device__ __forceinline__ void publish_aggregate(uint64_t *index, uint64_t t, uint64_t agg,
+                                                  bool bad) {
+    st_relaxed_u64(&index[t], (t == 0 ? FLAG_P : FLAG_A) | (bad ? BIT_RANGE : 0) | agg);
+}
+
+struct LookbackWindow {
+    uint64_t d[LB_PER_LANE];
+};
+
+__device__ __forceinline__ void lookback_issue(const uint64_t *index, int64_t j, LookbackWindow &w) {
+    const int64_t base = j - (threadIdx.x & 31) * LB_PER_LANE;
+#pragma unroll
+    for (int u = 0; u < LB_PER_LANE; u++)
+        w.d[u] = (base - u >= 0) ? ld_relaxed_u64(&index[base - u]) : FLAG_P;  // virtual P|0
+}
+
+// Returns the exclusive prefix of tile t (>= 1) and publishes its inclusive
+// descriptor; *range_out = RANGE bit of the inclusive prefix.
+__device__ __forceinline__ uint64_t lookback_finish(uint64_t *index, uint64_t t, uint64_t agg,
+                                                    bool bad, LookbackWindow &w, bool *range_out) {
     const int lane = threadIdx.x & 31;
-    if (t == 0) {
-        if (lane == 0) st_release_u64(&index[0], FLAG_P | agg);
-        return 0;
-    }
-    if (lane == 0) st_release_u64(&index[t], FLAG_A | agg);
-    uint64_t excl = 0;
-    int64_t j = static_cast<int64_t>(t) - 1;
-    while (true) {
-        const int64_t idx = j - lane;
-        uint64_t d = FLAG_P;  // virtual P|0 before tile 0
-        if (idx >= 0) {
-            d = ld_acquire_u64(&index[idx]);
-            while ((d >> 62) == 0) {  // Waiting: spin until published
-                __nanosleep(20);
-                d = ld_acquire_u64(&index[idx]);
+    uint64_t excl = 0, rbits = bad ? BIT_RANGE : 0;
+    int64_t j = static_cast<int64_t>(t) - 1;  // nearest predecessor of the window
+    bool done = false;
+    while (!done) {
+        const int64_t base = j - lane * LB_PER_LANE;
+        while (true) {
+            // lane-local walk, nearest first: st 2 = met a P, 1 = all A, 0 = met a Waiting slot
+            uint64_t sum = 0, rb = 0;
+            int st = 1;
+#pragma unroll
+            for (int u = 0; u < LB_PER_LANE; u++) {
+                if (st == 1) {
+                    const uint64_t f = w.d[u] >> 62;
+                    if (f == 0) {
+                        st = 0;
+                    } else {
+                        sum += w.d[u] & VAL61;
+                        rb |= w.d[u] & BIT_RANGE;
+                        if (f == 2) st = 2;
+                    }
+                }
             }
-        }
-        const unsigned pmask = __ballot_sync(0xffffffffu, (d >> 62) == 2);
-        uint64_t v = d & VAL_MASK;
-        if (pmask) {
-            const int p = __ffs(pmask) - 1;  // nearest predecessor with a prefix
-            excl += warp_sum_u64(lane <= p ? v : 0);
+            const unsigned pm = __ballot_sync(0xffffffffu, st == 2);
+            const unsigned wm = __ballot_sync(0xffffffffu, st == 0);
+            const int p = pm ? __ffs(pm) - 1 : 32;
+            const int wt = wm ? __ffs(wm) - 1 : 32;
+            if (wt < p) {  // a needed predecessor is still Waiting: re-poll the empty slots
+                __nanosleep(32);
+#pragma unroll
+                for (int u = 0; u < LB_PER_LANE; u++)
+                    if (base - u >= 0 && (w.d[u] >> 62) == 0) w.d[u] = ld_relaxed_u64(&index[base - u]);
+                continue;
+            }
+            excl += warp_sum_u64(lane <= p ? sum : 0);
+            rbits |= __ballot_sync(0xffffffffu, lane <= p && rb != 0) ? BIT_RANGE : 0;
+            done = p < 32;
             break;
         }
-        excl += warp_sum_u64(v);
-        j -= 32;
+        if (!done) {
+            j -= 32 * LB_PER_LANE;
+            lookback_issue(index, j, w);
+        }
     }
-    if (lane == 0) st_release_u64(&index[t], FLAG_P | (excl + agg));
+    if (lane == 0) st_relaxed_u64(&index[t], FLAG_P | rbits | (excl + agg));
+    *range_out = rbits != 0;
     return excl;
 }
 
@@ -346,234 +395,341 @@ struct HdrStatic {
     double eb_user;    // header bytes 24..31
 };
 
+// Three rotating tile buffers per CTA: tile i is encoded out of one (and its
+// payload staged back into it), tile i-1's staged payload waits in another for its
+// prefix, and tile i+1 streams into the third.
+constexpr int NBUF = 3;
+template <typename T>
+struct CompLayout {
+    static constexpr uint32_t STRIDE = Traits<T>::TILE_BYTES + (sizeof(T) == 4 ? 1024 : 0);
+    static constexpr int SMEM = NBUF * STRIDE + 1024;
+};
 template <typename T>
 constexpr int compress_smem_bytes() {
-    return Traits<T>::TILE_BYTES + 1024 + 128;
+    return CompLayout<T>::SMEM;
 }
 
+// Copy a tile's staged payload (smem, tile-relative, 16-byte aligned base) to its
+// global byte range [dst0, dst0 + bytes): 16-byte aligned chunks by coalesced
+// 128-bit stores (funnel-shifted out of smem), the unaligned head/tail by bytes.
+__device__ __forceinline__ void write_payload(const uint8_t *stg, uint8_t *out, uint64_t dst0,
+                                              uint32_t bytes) {
+    const int tid = threadIdx.x;
+    const uint64_t dst1 = dst0 + bytes;
+    const uint64_t a0 = roundup16(dst0), a1 = dst1 & ~uint64_t(15);
+    if (a0 < a1) {
+        const uint32_t s0 = static_cast<uint32_t>(a0 - dst0);  // 0..15
+        const uint32_t sh = 8u * (s0 & 3u);
+        const uint32_t *sw = reinterpret_cast<const uint32_t *>(stg) + (s0 >> 2);
+        const uint32_t nchunks = static_cast<uint32_t>((a1 - a0) >> 4);
+        for (uint32_t c = tid; c < nchunks; c += NT) {
+            const uint32_t *w = sw + 4 * c;
+            const uint32_t v0 = w[0], v1 = w[1], v2 = w[2], v3 = w[3], v4 = w[4];
+            uint4 o;
+            o.x = __funnelshift_r(v0, v1, sh);
+            o.y = __funnelshift_r(v1, v2, sh);
+            o.z = __funnelshift_r(v2, v3, sh);
+            o.w = __funnelshift_r(v3, v4, sh);
+            *reinterpret_cast<uint4 *>(out + a0 + 16ull * c) = o;
+        }
+        if (tid >= NT - 32 && tid < NT - 16) {  // head bytes
+            const uint64_t o = dst0 + (tid - (NT - 32));
+            if (o < a0) out[o] = stg[o - dst0];
+        } else if (tid >= NT - 16) {  // tail bytes
+            const uint64_t o = a1 + (tid - (NT - 16));
+            if (o < dst1) out[o] = stg[o - dst0];
+        }
+    } else if (tid >= NT - 32) {  // the whole payload is < 32 bytes
+        const uint64_t o = dst0 + (tid - (NT - 32));
+        if (o < dst1) out[o] = stg[o - dst0];
+    }
+}
+
+// Persistent compression kernel. Tiles are claimed in order from an atomic
+// ticket (every predecessor a lookback waits for belongs to a running CTA) and
+// loaded by TMA one tile ahead. Iteration i: encode tile i (❶ ❷, payload staged in
+// smem at tile-relative offsets), publish its aggregate, claim + prefetch tile
+// i+1, then resolve the prefix of tile i-1 (❸) — by now usually one L2 round trip —
+// and write tile i-1 out (❹). A claimed tile is never held behind a lookback wait,
+// which would serialise the whole machine on the P frontier.
 template <typename T, bool OUTLIER>
-__global__ void __launch_bounds__(NT) compress_kernel(const __grid_constant__ CUtensorMap tmap,
-                                                      const T *__restrict__ in, const Geom g,
-                                                      const double eb_abs_arg,
-                                                      const int eb_from_header,
-                                                      uint8_t *__restrict__ out,
-                                                      uint64_t *__restrict__ d_out_bytes,
-                                                      const HdrStatic hs) {
+__global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) compress_kernel(
+    const __grid_constant__ CUtensorMap tmap, const T *__restrict__ in, const Geom g,
+    const double eb_abs_arg, const int eb_from_header, uint8_t *__restrict__ out,
+    unsigned *__restrict__ ticket, uint64_t *__restrict__ d_out_bytes, const HdrStatic hs) {
     extern __shared__ uint8_t smem_raw[];
-    uint8_t *tile = reinterpret_cast<uint8_t *>(
+    constexpr uint32_t STRIDE = CompLayout<T>::STRIDE;
+    uint8_t *bufs = reinterpret_cast<uint8_t *>(
         (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    __shared__ uint64_t s_bar;
-    __shared__ uint32_t s_ticket;
+    __shared__ uint64_t s_bar[NBUF];
+    __shared__ uint32_t s_tk[NBUF];
     __shared__ uint32_t s_warp[NT / 32];
-    __shared__ uint64_t s_tile_excl;
+    __shared__ uint64_t s_excl;
+    __shared__ bool s_rng;
 
     const int tid = threadIdx.x;
     const uint64_t T_eff = g.T ? g.T : 1;
+    uint64_t *index = reinterpret_cast<uint64_t *>(out + 64);
 
-    if (tid == 0) {
-        // dynamic tile id: tiles are handed out in order, so every predecessor a
-        // lookback waits for is already resident (forward progress)
-        s_ticket = atomicAdd(reinterpret_cast<unsigned *>(out + 56), 1u);
-        mbar_init(&s_bar, 1);
+    // TMA thread: start the load of tile `tk` into buffer `bi` (always arrives on
+    // the buffer's mbarrier so its phase advances even without data)
+    auto issue = [&](uint64_t tk, int bi) {
+        uint64_t *bar = &s_bar[bi];
+        uint8_t *dst = bufs + bi * STRIDE;
+        const uint64_t b0 = tk * BPT;
+        if (tk < T_eff && b0 < g.nfull) {
+            if (Traits<T>::ROWS == 1) {
+                mbar_expect_tx(bar, BPT * 128);
+                tma_load_2d(dst, &tmap, 0, static_cast<int>(b0), bar);
+            } else {
+                const bool second = (b0 + BPT / 2) < g.nfull;
+                mbar_expect_tx(bar, second ? 2 * BPT * 128 : BPT * 128);
+                tma_load_2d(dst, &tmap, 0, static_cast<int>(2 * b0), bar);
+                if (second) tma_load_2d(dst + BPT * 128, &tmap, 0, static_cast<int>(2 * b0 + BPT), bar);
+            }
+        } else {
+            mbar_expect_tx(bar, 0);
+        }
+    };
+
+    if (tid == TMA_TID) {
+        for (int i = 0; i < NBUF; i++) mbar_init(&s_bar[i], 1);
         fence_mbar_init();
+        const uint32_t tk = atomicAdd(ticket, 1u);
+        s_tk[0] = tk;
+        issue(tk, 0);
     }
     __syncthreads();
-    const uint64_t t = s_ticket;
-    const uint64_t b0 = t * BPT;
-    const bool has_rows = b0 < g.nfull;
-    if (tid == 0 && has_rows) {
-        if (Traits<T>::ROWS == 1) {
-            mbar_expect_tx(&s_bar, BPT * 128);
-            tma_load_2d(tile, &tmap, 0, static_cast<int>(b0), &s_bar);
-        } else {
-            const bool second = (b0 + BPT / 2) < g.nfull;
-            mbar_expect_tx(&s_bar, second ? 2 * BPT * 128 : BPT * 128);
-            tma_load_2d(tile, &tmap, 0, static_cast<int>(2 * b0), &s_bar);
-            if (second)
-                tma_load_2d(tile + BPT * 128, &tmap, 0, static_cast<int>(2 * b0 + BPT), &s_bar);
-        }
-    }
 
     // constants of the arithmetic contract (FORMAT.md §6.2)
     const double eb_abs =
         eb_from_header ? *reinterpret_cast<const volatile double *>(out + 32) : eb_abs_arg;
     const auto K = make_consts(eb_abs, static_cast<T *>(nullptr));
 
-    const uint64_t b = b0 + tid;
-    const bool active = b < g.nb;
-    const bool full = b < g.nfull;
+    uint64_t prev_t = ~uint64_t(0);  // tile encoded in the previous iteration (uniform)
+    uint32_t prev_agg = 0;
+    bool prev_bad = false;
+    LookbackWindow win;
+    for (uint32_t it = 0;; ++it) {
+        const int cur = it % NBUF;
+        const uint64_t t = s_tk[cur];
+        const bool have_cur = t < T_eff;
+        const bool have_prev = prev_t != ~uint64_t(0);
+        if (!have_cur && !have_prev) break;
+        const bool do_lookback = have_prev && g.T && prev_t > 0;
+        if (do_lookback && tid < 32)  // predecessors' descriptors fly while this tile encodes
+            lookback_issue(index, static_cast<int64_t>(prev_t) - 1, win);
 
-    if (has_rows) mbar_wait(&s_bar, 0);
+        uint32_t agg = 0;
+        bool any_bad = false;
+        if (have_cur) {
+            uint8_t *tile = bufs + cur * STRIDE;
+            const uint64_t b = t * BPT + tid;
+            const bool active = b < g.nb;
+            const bool full = b < g.nfull;
+            mbar_wait(&s_bar[cur], (it / NBUF) & 1);
 
-    // ---- load the block's 32 values
-    T x[L];
-    uint32_t valid = L;
-    if (full) {
-        load_block(tile, tid, x);
-    } else {
-        valid = active ? static_cast<uint32_t>(g.n - b * L) : 0u;
+            // ---- load the block's 32 values
+            T x[L];
+            uint32_t valid = L;
+            if (full) {
+                load_block(tile, tid, x);
+            } else {
+                valid = active ? static_cast<uint32_t>(g.n - b * L) : 0u;
 #pragma unroll
-        for (int i = 0; i < L; i++) x[i] = (i < (int)valid) ? in[b * L + i] : T(0);
-    }
+                for (int i = 0; i < L; i++) x[i] = (i < (int)valid) ? in[b * L + i] : T(0);
+            }
 
-    // ---- ❶ pre-quantization + in-block first-order difference
-    bool bad = false;
-    int q[L];
+            // ---- ❶ pre-quantization + in-block first-order difference
+            bool bad = false;
+            int q[L];
 #pragma unroll
-    for (int i = 0; i < L; i++) q[i] = quantize(x[i], K.inv, bad);
-    if (!full) {  // tail block: q_i = q_{i-1} past n (FORMAT.md §6.4)
+            for (int i = 0; i < L; i++) q[i] = quantize(x[i], K.inv, bad);
+            if (!full) {  // tail block: q_i = q_{i-1} past n (FORMAT.md §6.4)
 #pragma unroll
-        for (int i = 1; i < L; i++)
-            if (i >= (int)valid) q[i] = q[i - 1];
-    }
-    uint32_t a[L];
-    uint32_t sign = 0, or_rest = 0;
+                for (int i = 1; i < L; i++)
+                    if (i >= (int)valid) q[i] = q[i - 1];
+            }
+            uint32_t a[L];
+            uint32_t sign = 0, or_rest = 0;
 #pragma unroll
-    for (int i = 0; i < L; i++) {
-        const int d = q[i] - (i ? q[i - 1] : 0);
-        a[i] = static_cast<uint32_t>(d < 0 ? -d : d);
-        sign |= static_cast<uint32_t>(d < 0) << i;
-        if (i) or_rest |= a[i];
-    }
+            for (int i = 0; i < L; i++) {
+                const int d = q[i] - (i ? q[i - 1] : 0);
+                a[i] = static_cast<uint32_t>(d < 0 ? -d : d);
+                sign |= static_cast<uint32_t>(d < 0) << i;
+                if (i) or_rest |= a[i];
+            }
 
-    // ---- ❷ fixed lengths and the fine-tuned Plain/Outlier selection
-    const int fl_p = 32 - __clz(or_rest | a[0]);
-    uint32_t size = fl_p ? 4u * (1u + fl_p) : 0u;
-    uint32_t obyte = static_cast<uint32_t>(fl_p);
-    int fl = fl_p, nob = 0;
-    if (OUTLIER) {
-        const int fl_o = 32 - __clz(or_rest);
-        const int ob = max(1, (32 - __clz(a[0]) + 7) >> 3);
-        const uint32_t size_o = 4u + ob + 4u * fl_o;
-        if (size_o < size) {
-            size = size_o;
-            obyte = 0x80u | (static_cast<uint32_t>(ob - 1) << 5) | static_cast<uint32_t>(fl_o);
-            fl = fl_o;
-            nob = ob;
-        }
-    }
-    if (!active) {
-        size = 0;
-        bad = false;
-    }
-    if (!K.ok) bad = true;
+            // ---- ❷ fixed lengths and the fine-tuned Plain/Outlier selection
+            const int fl_p = 32 - __clz(or_rest | a[0]);
+            uint32_t size = fl_p ? 4u * (1u + fl_p) : 0u;
+            uint32_t obyte = static_cast<uint32_t>(fl_p);
+            int fl = fl_p, nob = 0;
+            if (OUTLIER) {
+                const int fl_o = 32 - __clz(or_rest);
+                const int ob = max(1, (32 - __clz(a[0]) + 7) >> 3);
+                const uint32_t size_o = 4u + ob + 4u * fl_o;
+                if (size_o < size) {
+                    size = size_o;
+                    obyte = 0x80u | (static_cast<uint32_t>(ob - 1) << 5) | static_cast<uint32_t>(fl_o);
+                    fl = fl_o;
+                    nob = ob;
+                }
+            }
+            if (!active) {
+                size = 0;
+                bad = false;
+            }
+            if (!K.ok) bad = true;
 
-    // ---- ❸ intra-tile scan + decoupled lookback across tiles
-    const bool any_bad = __syncthreads_or(bad);
-    uint32_t agg;
-    const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg);
-    if (tid < 32) {
-        if (any_bad && tid == 0)  // status before the descriptor is released
-            atomicOr(reinterpret_cast<unsigned *>(out + 8), static_cast<unsigned>(ST_RANGE) << 8);
-        uint64_t excl = 0;
-        if (g.T) excl = lookback(reinterpret_cast<uint64_t *>(out + 64), t, agg);
-        if (tid == 0) s_tile_excl = excl;
-    }
+            // ---- intra-tile scan ("Reduce"); every thread is done reading `tile` after it
+            any_bad = __syncthreads_or(bad);
+            const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg);
+            if (tid == 0 && g.T) publish_aggregate(index, t, agg, any_bad);
+            if (tid == TMA_TID) {  // claim + prefetch the next tile right behind the publish
+                const int nxt = (it + 1) % NBUF;
+                const uint32_t tn = atomicAdd(ticket, 1u);
+                s_tk[nxt] = tn;
+                if (tn < T_eff) issue(tn, nxt);
+            }
+            if (active) out[g.O + b] = static_cast<uint8_t>(obyte);  // ❹ offset bytes
 
-    // ---- ❹ concatenation: offset byte straight to global, payload staged in smem
-    if (active) out[g.O + b] = static_cast<uint8_t>(obyte);
-    __syncthreads();  // s_tile_excl visible; every thread is done reading `tile`
-    const uint64_t tile_excl = s_tile_excl;
-    const uint64_t dst0 = g.D + tile_excl;
-    const uint32_t phase = static_cast<uint32_t>(dst0 & 15u);
-    if (size) {
-        uint8_t *p = tile + phase + my_excl;
-        st_u32_unaligned(p, sign);
-        p += 4;
-        if (OUTLIER && nob) {
-            for (int j = 0; j < nob; j++) p[j] = static_cast<uint8_t>(a[0] >> (8 * j));
-            p += nob;
-            a[0] = 0;  // the outlier slot of every plane is 0
-        }
-        if (fl) {
-            const int sh = 32 - fl;
+            // ---- ❷ payload staged at its tile-relative byte offset
+            if (size) {
+                uint8_t *p = tile + my_excl;
+                st_u32_unaligned(p, sign);
+                p += 4;
+                if (OUTLIER && nob) {
+                    for (int j = 0; j < nob; j++) p[j] = static_cast<uint8_t>(a[0] >> (8 * j));
+                    p += nob;
+                    a[0] = 0;  // the outlier slot of every plane is 0
+                }
+                if (fl) {
+                    const int sh = 32 - fl;
 #pragma unroll
-            for (int i = 0; i < L; i++) a[i] <<= sh;
-            for (int k = fl - 1; k >= 0; k--) {  // planes top-down, 2 ops per bit
-                uint32_t w = 0;
+                    for (int i = 0; i < L; i++) a[i] <<= sh;
+                    for (int k = fl - 1; k >= 0; k--) {  // planes top-down, 2 ops per bit
+                        uint32_t w = 0;
 #pragma unroll
-                for (int i = L - 1; i >= 0; i--) shift_bit_into(a[i], w);
-                st_u32_unaligned(p + 4 * k, w);
+                        for (int i = L - 1; i >= 0; i--) shift_bit_into(a[i], w);
+                        st_u32_unaligned(p + 4 * k, w);
+                    }
+                }
             }
         }
-    }
-    fence_proxy_async_smem();
-    __syncthreads();
 
-    const uint64_t dst1 = dst0 + agg;
-    const uint64_t m0 = roundup16(dst0), m1 = dst1 & ~uint64_t(15);
-    if (m0 < m1) {
-        if (tid == 0) {
-            bulk_store(out + m0, tile + (m0 - (dst0 & ~uint64_t(15))), static_cast<uint32_t>(m1 - m0));
-            bulk_commit();
+        if (have_prev) {
+            // ---- ❸ prefix of the previous tile, then ❹ its payload to global
+            if (tid < 32) {
+                bool rng = prev_bad;
+                const uint64_t e =
+                    do_lookback ? lookback_finish(index, prev_t, prev_agg, prev_bad, win, &rng) : 0;
+                if (tid == 0) {
+                    s_excl = e;
+                    s_rng = rng;
+                }
+            }
+            __syncthreads();
+            const uint64_t excl = s_excl;
+            const uint8_t *stg = bufs + ((it + NBUF - 1) % NBUF) * STRIDE;
+            const uint64_t dst0 = g.D + excl;
+            write_payload(stg, out, dst0, prev_agg);
+            if (prev_t == T_eff - 1) {  // last tile: pads, header, d_out_bytes
+                const uint64_t dst1 = dst0 + prev_agg;
+                if (tid >= 32 && tid < 48) {  // zero pad after the payload
+                    const uint64_t o = dst1 + (tid - 32);
+                    if (o < roundup16(dst1)) out[o] = 0;
+                }
+                if (tid >= 64 && tid < 80) {  // zero pad after the offset bytes
+                    const uint64_t o = g.O + g.nb + (tid - 64);
+                    if (o < g.D) out[o] = 0;
+                }
+                if (tid == 0) {
+                    const uint32_t status = s_rng ? ST_RANGE : 0u;
+                    const uint64_t pb = status ? 0 : excl + prev_agg;
+                    const uint64_t total = roundup16(g.D + pb);
+                    uint64_t *h = reinterpret_cast<uint64_t *>(out);
+                    h[0] = MAGIC | (static_cast<uint64_t>(hs.word1) << 32);
+                    h[1] = hs.eb_mode | (status << 8) | (static_cast<uint64_t>(BPT) << 16);
+                    h[2] = g.n;
+                    h[3] = static_cast<uint64_t>(__double_as_longlong(hs.eb_user));
+                    h[4] = static_cast<uint64_t>(__double_as_longlong(eb_abs));
+                    h[5] = pb;
+                    h[6] = total;
+                    h[7] = 0;
+                    if (d_out_bytes) *d_out_bytes = total;
+                }
+            }
         }
-        if (tid >= 32 && tid < 48) {  // unaligned head bytes
-            const uint64_t o = dst0 + (tid - 32);
-            if (o < m0) out[o] = tile[phase + (o - dst0)];
-        }
-        if (tid >= 64 && tid < 80) {  // unaligned tail bytes
-            const uint64_t o = m1 + (tid - 64);
-            if (o < dst1) out[o] = tile[phase + (o - dst0)];
-        }
-    } else if (tid >= 96 && tid < 128) {  // whole tile payload < 32 bytes
-        const uint64_t o = dst0 + (tid - 96);
-        if (o < dst1) out[o] = tile[phase + (o - dst0)];
+        if (!have_cur) break;  // the previous tile was the last one this CTA held
+        prev_t = t;
+        prev_agg = agg;
+        prev_bad = any_bad;
+        __syncthreads();  // staging reads done before the buffer is refilled; s_tk visible
     }
-
-    if (t == T_eff - 1) {  // last tile: pads, header, d_out_bytes
-        if (tid >= 128 && tid < 144) {  // zero pad after the payload
-            const uint64_t o = dst1 + (tid - 128);
-            if (o < roundup16(dst1)) out[o] = 0;
-        }
-        if (tid >= 160 && tid < 176) {  // zero pad after the offset bytes
-            const uint64_t o = g.O + g.nb + (tid - 160);
-            if (o < g.D) out[o] = 0;
-        }
-        if (tid == 0) {
-            const uint32_t w8 = ld_acquire_u32(reinterpret_cast<const uint32_t *>(out + 8));
-            const uint32_t status = (w8 >> 8) & 0xFFu;
-            const uint64_t pb = status ? 0 : tile_excl + agg;
-            const uint64_t total = roundup16(g.D + pb);
-            uint64_t *h = reinterpret_cast<uint64_t *>(out);
-            h[0] = MAGIC | (static_cast<uint64_t>(hs.word1) << 32);
-            h[1] = hs.eb_mode | (status << 8) | (static_cast<uint64_t>(BPT) << 16);
-            h[2] = g.n;
-            h[3] = static_cast<uint64_t>(__double_as_longlong(hs.eb_user));
-            h[4] = static_cast<uint64_t>(__double_as_longlong(eb_abs));
-            h[5] = pb;
-            h[6] = total;
-            h[7] = 0;
-            if (d_out_bytes) *d_out_bytes = total;
-        }
-    }
-    if (tid == 0 && m0 < m1) bulk_wait0();
 }
 
 // ------------------------------------------------------------------ decompression
-template <typename T>
-constexpr int decompress_smem_bytes() {
-    return Traits<T>::TILE_BYTES + BPT * 4 * L + 64 + 1024 + 128;
-}
+constexpr uint32_t PBUF_BYTES = BPT * 4 * L + 128;  // max tile payload + alignment slack
 
 template <typename T>
-__global__ void __launch_bounds__(NT) decompress_kernel(const __grid_constant__ CUtensorMap tmap,
-                                                        const uint8_t *__restrict__ cmp,
-                                                        T *__restrict__ out, const Geom g,
-                                                        int *__restrict__ d_status) {
+constexpr int decompress_smem_bytes() {
+    return Traits<T>::TILE_BYTES + 2 * PBUF_BYTES + 1024;
+}
+
+// Persistent decompression kernel: CTA c decodes tiles c, c+G, c+2G, ... The
+// persisted tile index locates every tile in O(1) (no inter-CTA waiting), so the
+// next tile's index words, offset bytes and payload (1D bulk TMA) are fetched
+// while the current tile is decoded and stored (2D tensor TMA, 128B swizzle).
+template <typename T>
+__global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) decompress_kernel(const __grid_constant__ CUtensorMap tmap,
+                                                           const uint8_t *__restrict__ cmp,
+                                                           T *__restrict__ out, const Geom g,
+                                                           int *__restrict__ d_status) {
     extern __shared__ uint8_t smem_raw[];
     uint8_t *ostage = reinterpret_cast<uint8_t *>(
         (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    uint8_t *pbuf = ostage + Traits<T>::TILE_BYTES;
-    __shared__ uint64_t s_bar;
+    uint8_t *pbufs = ostage + Traits<T>::TILE_BYTES;
+    __shared__ uint64_t s_bar[2];
     __shared__ uint32_t s_warp[NT / 32];
-    __shared__ uint64_t s_excl, s_bytes;
+    __shared__ uint64_t s_excl[2];
+    __shared__ uint32_t s_bytes[2];
     __shared__ double s_eb;
     __shared__ int s_err;
 
     const int tid = threadIdx.x;
-    const uint64_t t = blockIdx.x;
+    const uint64_t G = gridDim.x;
+    const uint64_t *index = reinterpret_cast<const uint64_t *>(cmp) + 8;
+    constexpr uint32_t BAD_BYTES = 0xFFFFFFFFu;
+
+    // thread 0 state: raw index words of the tile two steps ahead
+    uint64_t raw_p = FLAG_P, raw_i = 0;
+    uint64_t pb_hdr = 0;   // payload bytes from the header
+    bool pending = false;  // a payload prefetch is in flight
+
+    // thread 0: tile meta from two index words -> smem slot, start its payload TMA
+    auto launch = [&](uint64_t tt, uint64_t dp, uint64_t di, int bi) {
+        const uint64_t e = dp & VAL_MASK, i = di & VAL_MASK;  // bit 61 is 0 in a valid stream
+        uint32_t bytes = BAD_BYTES;
+        if ((dp >> 61) == 4 && (di >> 61) == 4 && i >= e && i <= pb_hdr &&
+            i - e <= static_cast<uint64_t>(BPT) * 4 * L)
+            bytes = static_cast<uint32_t>(i - e);
+        s_excl[bi] = e;
+        s_bytes[bi] = bytes;
+        if (bytes != BAD_BYTES && bytes) {
+            const uint64_t src0 = (g.D + e) & ~uint64_t(15);
+            const uint32_t len = static_cast<uint32_t>(roundup16(g.D + e + bytes) - src0);
+            mbar_expect_tx(&s_bar[bi], len);
+            bulk_load(pbufs + bi * PBUF_BYTES, cmp + src0, len, &s_bar[bi]);
+        } else {
+            mbar_expect_tx(&s_bar[bi], 0);
+        }
+        (void)tt;
+    };
+
+    uint64_t t = blockIdx.x;
     if (tid == 0) {
-        // header checks (FORMAT.md §3) — every CTA reads the 64 L2-resident bytes
+        // header checks (FORMAT.md §3) — once per CTA
         const uint64_t *h = reinterpret_cast<const uint64_t *>(cmp);
         const uint64_t h0 = h[0], h1 = h[1];
         int err = 0;
@@ -583,115 +739,145 @@ __global__ void __launch_bounds__(NT) decompress_kernel(const __grid_constant__ 
             err = ST_FORMAT;
         else if (((h1 >> 8) & 0xFF) != 0)
             err = ((h1 >> 8) & 0xFF) == ST_RANGE ? ST_RANGE : ST_FORMAT;
-        const uint64_t pb = h[5];
-        if (!err && h[6] != roundup16(g.D + pb)) err = ST_FORMAT;
-        uint64_t excl = 0, incl = 0;
-        if (!err && t < g.T) {
-            const uint64_t *index = h + 8;
-            const uint64_t dp = t ? index[t - 1] : FLAG_P;
-            const uint64_t di = index[t];
-            excl = dp & VAL_MASK;
-            incl = di & VAL_MASK;
-            if ((dp >> 62) != 2 || (di >> 62) != 2 || incl < excl || incl > pb ||
-                incl - excl > static_cast<uint64_t>(BPT) * 4 * L)
-                err = ST_FORMAT;
-        }
+        pb_hdr = h[5];
+        if (!err && h[6] != roundup16(g.D + pb_hdr)) err = ST_FORMAT;
         s_eb = __longlong_as_double(static_cast<long long>(h[4]));
-        s_excl = excl;
-        s_bytes = incl - excl;
         s_err = err;
-        mbar_init(&s_bar, 1);
+        mbar_init(&s_bar[0], 1);
+        mbar_init(&s_bar[1], 1);
         fence_mbar_init();
+        if (!err && t < g.T) {
+            launch(t, t ? index[t - 1] : FLAG_P, index[t], 0);
+            pending = true;
+            const uint64_t t2 = t + G;
+            if (t2 < g.T) {
+                raw_p = index[t2 - 1];
+                raw_i = index[t2];
+            }
+        }
     }
     __syncthreads();
-    if (s_err || t >= g.T) {
-        if (tid == 0 && s_err && d_status) atomicOr(d_status, s_err);
+    if (s_err) {
+        if (tid == 0 && d_status) atomicOr(d_status, s_err);
         return;
     }
-    const uint64_t excl = s_excl;
-    const uint32_t bytes = static_cast<uint32_t>(s_bytes);
-    const uint64_t src0 = (g.D + excl) & ~uint64_t(15);
-    const uint32_t phase = static_cast<uint32_t>((g.D + excl) & 15u);
-    if (tid == 0 && bytes) {  // ❸ located in O(1): fetch the tile's payload bytes
-        const uint32_t len = static_cast<uint32_t>(roundup16(g.D + excl + bytes) - src0);
-        mbar_expect_tx(&s_bar, len);
-        bulk_load(pbuf, cmp + src0, len, &s_bar);
-    }
-
-    const uint64_t b = t * BPT + tid;
-    const bool active = b < g.nb;
-    const uint32_t obyte = active ? cmp[g.O + b] : 0u;
-    const uint32_t fl = obyte & 31u;
-    const bool is_o = (obyte & 0x80u) != 0;
-    const uint32_t nob = is_o ? ((obyte >> 5) & 3u) + 1u : 0u;
-    bool bad = (!is_o && (obyte & 0x60u));
-    const uint32_t size = is_o ? 4u + nob + 4u * fl : (fl ? 4u * (1u + fl) : 0u);
-    uint32_t agg;
-    const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg);
-    bad |= (tid == 0 && agg != bytes);
-    if (__syncthreads_or(bad)) {
-        if (tid == 0) {
-            if (bytes) mbar_wait(&s_bar, 0);  // never exit with a bulk copy in flight
-            if (d_status) atomicOr(d_status, ST_FORMAT);
-        }
-        return;
-    }
-    if (bytes) mbar_wait(&s_bar, 0);
-
-    // ---- ❷⁻¹ decode: sign field, outlier, bit planes (top plane first)
-    uint32_t a[L];
-#pragma unroll
-    for (int i = 0; i < L; i++) a[i] = 0;
-    uint32_t sign = 0;
-    if (size) {
-        uint32_t pos = phase + my_excl;
-        sign = ld_u32_unaligned(pbuf, pos);
-        pos += 4;
-        uint32_t outlier = 0;
-        if (is_o) {
-            outlier = ld_u32_unaligned(pbuf, pos);
-            if (nob < 4) outlier &= (1u << (8 * nob)) - 1u;
-            pos += nob;
-        }
-        for (int k = static_cast<int>(fl) - 1; k >= 0; k--) {
-            uint32_t w = ld_u32_unaligned(pbuf, pos + 4 * k);
-#pragma unroll
-            for (int i = L - 1; i >= 0; i--) shift_bit_into(w, a[i]);
-        }
-        if (is_o) a[0] = outlier;
-    }
-    // ---- inverse Lorenzo (prefix sum) + ❶⁻¹ dequantization
     const auto K = make_consts(s_eb, static_cast<T *>(nullptr));
-    T x[L];
-    int qv = 0;
-#pragma unroll
-    for (int i = 0; i < L; i++) {
-        const int d = ((sign >> i) & 1u) ? -static_cast<int>(a[i]) : static_cast<int>(a[i]);
-        qv += d;
-        x[i] = dequantize(qv, K.s);
+    uint32_t ob_cur = 0, ob_next = 0;
+    {
+        const uint64_t b = t * BPT + tid;
+        if (t < g.T && b < g.nb) ob_cur = cmp[g.O + b];
+        const uint64_t bn = (t + G) * BPT + tid;
+        if (t + G < g.T && bn < g.nb) ob_next = cmp[g.O + bn];
     }
-    const bool full = b < g.nfull;
-    if (full) {
-        store_block(ostage, tid, x);
-    } else if (active) {  // ragged tail block: only valid values
-        const uint32_t valid = static_cast<uint32_t>(g.n - b * L);
-#pragma unroll
-        for (int i = 0; i < L; i++)
-            if (i < (int)valid) out[b * L + i] = x[i];
-    }
-    fence_proxy_async_smem();
-    __syncthreads();
-    const uint64_t b0 = t * BPT;
-    if (tid == 0 && b0 < g.nfull) {
-        if (Traits<T>::ROWS == 1) {
-            tma_store_2d(&tmap, 0, static_cast<int>(b0), ostage);
-        } else {
-            tma_store_2d(&tmap, 0, static_cast<int>(2 * b0), ostage);
-            if (b0 + BPT / 2 < g.nfull)
-                tma_store_2d(&tmap, 0, static_cast<int>(2 * b0 + BPT), ostage + BPT * 128);
+
+    int err = 0;
+    for (uint32_t it = 0; t < g.T; ++it, t += G) {
+        const int cur = it & 1;
+        const uint64_t tn = t + G;
+        if (tid == 0) {
+            pending = false;
+            if (tn < g.T) {  // payload of the next tile streams in during this one
+                launch(tn, raw_p, raw_i, cur ^ 1);
+                pending = true;
+                const uint64_t t2 = tn + G;
+                if (t2 < g.T) {
+                    raw_p = index[t2 - 1];
+                    raw_i = index[t2];
+                }
+            }
         }
-        bulk_commit();
-        bulk_wait0();
+        uint32_t ob_pref = 0;  // offset byte of tile t + 2G, consumed two steps later
+        {
+            const uint64_t t2 = tn + G;
+            const uint64_t b2 = t2 * BPT + tid;
+            if (t2 < g.T && b2 < g.nb) ob_pref = cmp[g.O + b2];
+        }
+
+        const uint64_t b0 = t * BPT;
+        const uint64_t b = b0 + tid;
+        const bool active = b < g.nb;
+        const uint32_t obyte = ob_cur;
+        const uint32_t fl = obyte & 31u;
+        const bool is_o = (obyte & 0x80u) != 0;
+        const uint32_t nob = is_o ? ((obyte >> 5) & 3u) + 1u : 0u;
+        bool bad = (!is_o && (obyte & 0x60u));
+        const uint32_t size = is_o ? 4u + nob + 4u * fl : (fl ? 4u * (1u + fl) : 0u);
+        uint32_t agg;
+        const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg);
+        const uint32_t bytes = s_bytes[cur];
+        bad |= (tid == 0 && agg != bytes);
+        if (__syncthreads_or(bad)) {
+            err = ST_FORMAT;
+            if (tid == 0) {
+                mbar_wait(&s_bar[cur], (it >> 1) & 1);
+                if (pending) mbar_wait(&s_bar[cur ^ 1], ((it + 1) >> 1) & 1);
+            }
+            break;
+        }
+        mbar_wait(&s_bar[cur], (it >> 1) & 1);
+
+        // ---- ❷⁻¹ decode: sign field, outlier, bit planes (top plane first)
+        const uint8_t *pbuf = pbufs + cur * PBUF_BYTES;
+        const uint32_t phase = static_cast<uint32_t>((g.D + s_excl[cur]) & 15u);
+        uint32_t a[L];
+#pragma unroll
+        for (int i = 0; i < L; i++) a[i] = 0;
+        uint32_t sign = 0;
+        if (size) {
+            uint32_t pos = phase + my_excl;
+            sign = ld_u32_unaligned(pbuf, pos);
+            pos += 4;
+            uint32_t outlier = 0;
+            if (is_o) {
+                outlier = ld_u32_unaligned(pbuf, pos);
+                if (nob < 4) outlier &= (1u << (8 * nob)) - 1u;
+                pos += nob;
+            }
+            for (int k = static_cast<int>(fl) - 1; k >= 0; k--) {
+                uint32_t w = ld_u32_unaligned(pbuf, pos + 4 * k);
+#pragma unroll
+                for (int i = L - 1; i >= 0; i--) shift_bit_into(w, a[i]);
+            }
+            if (is_o) a[0] = outlier;
+        }
+        // ---- inverse Lorenzo (prefix sum) + ❶⁻¹ dequantization
+        T x[L];
+        int qv = 0;
+#pragma unroll
+        for (int i = 0; i < L; i++) {
+            const int d = ((sign >> i) & 1u) ? -static_cast<int>(a[i]) : static_cast<int>(a[i]);
+            qv += d;
+            x[i] = dequantize(qv, K.s);
+        }
+        if (tid == 0) bulk_wait_read0();  // the previous tile's store has read ostage
+        __syncthreads();
+        const bool full = b < g.nfull;
+        if (full) {
+            store_block(ostage, tid, x);
+        } else if (active) {  // ragged tail block: only valid values
+            const uint32_t valid = static_cast<uint32_t>(g.n - b * L);
+#pragma unroll
+            for (int i = 0; i < L; i++)
+                if (i < (int)valid) out[b * L + i] = x[i];
+        }
+        fence_proxy_async_smem();
+        __syncthreads();
+        if (tid == 0 && b0 < g.nfull) {
+            if (Traits<T>::ROWS == 1) {
+                tma_store_2d(&tmap, 0, static_cast<int>(b0), ostage);
+            } else {
+                tma_store_2d(&tmap, 0, static_cast<int>(2 * b0), ostage);
+                if (b0 + BPT / 2 < g.nfull)
+                    tma_store_2d(&tmap, 0, static_cast<int>(2 * b0 + BPT), ostage + BPT * 128);
+            }
+            bulk_commit();
+        }
+        ob_cur = ob_next;
+        ob_next = ob_pref;
+    }
+    if (tid == 0) {
+        bulk_wait_read0();
+        if (err && d_status) atomicOr(d_status, err);
     }
 }
 

@@ -17,7 +17,7 @@ if [[ $WHAT == ncu || $WHAT == all ]]; then
       --log-file $OUT/launches_$TAG.csv python bench.py --steps 2 --warmup 3 --no-plain --e2e-steps 1 \
       --cpu-sample-log2 16 > $OUT/ncu_list_$TAG.log 2>&1; echo "ncu list rc=$?"
   for K in compress_kernel decompress_kernel minmax_kernel; do
-    timeout 900 ncu --set full --clock-control none --import-source on -k regex:"^.*$K" -s 3 -c 1 \
+    timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base function -k regex:"^$K"  -s 3 -c 1 \
         -o $OUT/prof_${K}_$TAG -f python bench.py --steps 1 --warmup 3 --no-plain --e2e-steps 1 \
         --cpu-sample-log2 16 > $OUT/ncu_full_${K}_$TAG.log 2>&1; echo "ncu full $K rc=$?"
   done

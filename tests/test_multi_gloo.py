@@ -1,0 +1,93 @@
+"""World-size-2 gloo tests of the N>1 host logic (CPU, no GPU): slab partition,
+the all-gather of compressed sizes, container offsets, and that the per-rank
+streams' offset bytes / payloads concatenate to the single-stream ones
+(block independence). The per-slab compressor here is the oracle
+(test infrastructure); the CUDA path runs the same logic in bench.py."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from tests import streamparse as sp
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, n, eb, enc, result_q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        from paper_conf_sc_huangdlc24_b200.multi import gather_sizes, slab
+        from synthetic import make_field
+
+        s0, cnt = slab(n, world, rank)
+        x = make_field("cfg2", "cpu", s0, cnt).numpy()
+        s, rc = oracle.compress(x, eb, oracle.ABS, enc)
+        sizes = gather_sizes(torch.tensor([s.size], dtype=torch.int64))
+        offsets = np.concatenate([[0], np.cumsum(sizes.numpy())])
+        streams = [None] * world
+        dist.all_gather_object(streams, s.tobytes())
+        result_q.put((rank, s0, cnt, rc, sizes.tolist(), offsets.tolist(), streams if rank == 0 else None))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("enc", [0, 1])
+def test_two_rank_slabs_concatenate_to_single_stream(orc, enc):
+    world, n, eb = 2, 3 * 8192 + 32 * 7 + 5, 1e-3
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, n, eb, enc, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted([q.get(timeout=120) for _ in range(world)])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    # slabs: contiguous, block-aligned, cover [0, n)
+    assert res[0][1] == 0 and res[0][1] + res[0][2] == res[1][1] and res[1][1] + res[1][2] == n
+    assert res[1][1] % 32 == 0
+    assert all(r[3] == orc.OK for r in res)
+    streams = [np.frombuffer(b, np.uint8) for b in res[0][6]]
+    sizes = res[0][4]
+    assert sizes == [s.size for s in streams] and res[1][4] == sizes  # every rank sees the same sizes
+    assert res[0][5] == [0, sizes[0], sizes[0] + sizes[1]]
+    # block independence: per-rank offset bytes and payloads concatenate to the P=1 stream's
+    from synthetic import make_field
+
+    full, _ = orc.compress(make_field("cfg2", "cpu", 0, n).numpy(), eb, orc.ABS, enc)
+    pf = sp.parse(full)
+    parts = [sp.parse(s) for s in streams]
+    np.testing.assert_array_equal(np.concatenate([p["offsets"] for p in parts]), pf["offsets"])
+    _, _, _, D = pf["geometry"]
+    pay = lambda s, p: s[p["geometry"][3]:p["geometry"][3] + p["header"]["payload_bytes"]]
+    np.testing.assert_array_equal(np.concatenate([pay(s, p) for s, p in zip(streams, parts)]),
+                                  pay(full, pf))
+    np.testing.assert_array_equal(np.concatenate([p["q"] for p in parts]), pf["q"])
+
+
+def test_slab_edge_cases():
+    from paper_conf_sc_huangdlc24_b200.multi import slab
+
+    for n in (0, 1, 31, 33, 1000, 2**33):
+        for world in (1, 2, 4, 8):
+            spans = [slab(n, world, r) for r in range(world)]
+            assert spans[0][0] == 0
+            assert sum(c for _, c in spans) == n
+            for (a, c), (b, _) in zip(spans, spans[1:]):
+                assert a + c == b
+                assert b % 32 == 0 or b == n
+    assert slab(2**33, 8, 3) == (3 * 2**30, 2**30)
