@@ -92,10 +92,10 @@ int sm_count() {
 
 // persistent grid: every CTA resident (occupancy x SMs), never more than tiles
 template <typename K>
-unsigned persistent_grid(K kernel, int smem, uint64_t tiles, int *cache) {
+unsigned persistent_grid(K kernel, int threads, int smem, uint64_t tiles, int *cache) {
     if (*cache <= 0) {
         int per_sm = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, NT, smem) != cudaSuccess ||
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, smem) != cudaSuccess ||
             per_sm < 1)
             per_sm = 1;
         *cache = per_sm * sm_count();
@@ -134,7 +134,7 @@ int launch_compress(const void *d_in, const Geom &g, double eb, int eb_mode, int
     constexpr int smem = compress_smem_bytes<T>();
     std::call_once(once, [] { attr_rc = set_smem(compress_kernel<T, OUTLIER>, smem); });
     if (attr_rc) return attr_rc;
-    const unsigned grid = persistent_grid(compress_kernel<T, OUTLIER>, smem, g.T, &grid_cache);
+    const unsigned grid = persistent_grid(compress_kernel<T, OUTLIER>, NT_COMP, smem, g.T, &grid_cache);
     unsigned *ticket = reinterpret_cast<unsigned *>(static_cast<uint8_t *>(d_out) + stream_bound(g));
     CUtensorMap map;
     int rc = make_tmap(&map, d_in, Traits<T>::DTYPE, g.nfull);
@@ -144,7 +144,7 @@ int launch_compress(const void *d_in, const Geom &g, double eb, int eb_mode, int
                (static_cast<uint32_t>(enc_mode) << 16) | (5u << 24);
     hs.eb_mode = static_cast<uint32_t>(eb_mode);
     hs.eb_user = eb;
-    compress_kernel<T, OUTLIER><<<grid, NT, smem, st>>>(
+    compress_kernel<T, OUTLIER><<<grid, NT_COMP, smem, st>>>(
         map, static_cast<const T *>(d_in), g, eb, eb_mode == CSZP2_EB_REL ? 1 : 0,
         static_cast<uint8_t *>(d_out), ticket, d_out_bytes, hs);
     return launch_status();
@@ -159,7 +159,7 @@ int launch_decompress(const void *d_cmp, void *d_out, const Geom &g, int *d_stat
     constexpr int smem = decompress_smem_bytes<T>();
     std::call_once(once, [] { attr_rc = set_smem(decompress_kernel<T>, smem); });
     if (attr_rc) return attr_rc;
-    const unsigned grid = persistent_grid(decompress_kernel<T>, smem, g.T, &grid_cache);
+    const unsigned grid = persistent_grid(decompress_kernel<T>, NT, smem, g.T, &grid_cache);
     CUtensorMap map;
     int rc = make_tmap(&map, d_out, Traits<T>::DTYPE, g.nfull);
     if (rc) return rc;
@@ -173,6 +173,12 @@ int launch_decompress(const void *d_cmp, void *d_out, const Geom &g, int *d_stat
 extern "C" {
 
 const char *cszp2_version(void) { return "cszp2 1.0 sm_100a"; }
+
+#ifdef CSZP2_TRACE
+int cszp2_debug_set_trace(void *d_buf) {
+    return cudaMemcpyToSymbol(g_trace, &d_buf, sizeof(void *)) == cudaSuccess ? 0 : 2;
+}
+#endif
 
 uint64_t cszp2_compress_bound(uint64_t n, int dtype) {
     if (!wsize(dtype)) return 0;

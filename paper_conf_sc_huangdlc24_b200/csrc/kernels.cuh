@@ -21,6 +21,20 @@
 
 namespace cszp2 {
 
+#ifdef CSZP2_TRACE
+// debug build only: per-tile globaltimer stamps [claim, data, publishA, resolved, written, polls]
+__device__ uint64_t *g_trace = nullptr;
+__device__ __forceinline__ uint64_t gtimer() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+#define TRACE(tile, slot, val) \
+    do { if (g_trace) g_trace[(tile) * 8 + (slot)] = (val); } while (0)
+#else
+#define TRACE(tile, slot, val) do { } while (0)
+#endif
+
 constexpr int L = 32;      // values per block
 constexpr int BPT = 256;   // blocks per tile (FORMAT.md §1)
 constexpr int NT = 256;    // threads per CTA: one block per thread
@@ -162,10 +176,17 @@ __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
     return v;
 }
 
-// CTA-wide exclusive scan of one u32 per thread (NT = 256). Returns the
-// exclusive prefix; *total receives the sum. Contains two __syncthreads.
+// Exclusive scan of one u32 per thread over the NT threads 0..NT-1, synchronised
+// with barrier `bar_id` (0 = the whole CTA). Returns the exclusive prefix;
+// *total receives the sum. Contains two barriers.
+__device__ __forceinline__ void group_sync(uint32_t bar_id) {
+    if (bar_id == 0)
+        __syncthreads();
+    else
+        named_sync(bar_id, NT);
+}
 __device__ __forceinline__ uint32_t cta_exclusive_scan(uint32_t v, uint32_t *s_warp,
-                                                       uint32_t *total) {
+                                                       uint32_t *total, uint32_t bar_id = 0) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     uint32_t inc = v;
 #pragma unroll
@@ -174,7 +195,7 @@ __device__ __forceinline__ uint32_t cta_exclusive_scan(uint32_t v, uint32_t *s_w
         if (lane >= o) inc += y;
     }
     if (lane == 31) s_warp[warp] = inc;
-    __syncthreads();
+    group_sync(bar_id);
     uint32_t base = 0, tot = 0;
 #pragma unroll
     for (int w = 0; w < NT / 32; w++) {
@@ -183,7 +204,7 @@ __device__ __forceinline__ uint32_t cta_exclusive_scan(uint32_t v, uint32_t *s_w
         tot += s;
     }
     *total = tot;
-    __syncthreads();
+    group_sync(bar_id);
     return base + inc - v;
 }
 
@@ -253,6 +274,9 @@ __device__ __forceinline__ uint64_t lookback_finish(uint64_t *index, uint64_t t,
             const int p = pm ? __ffs(pm) - 1 : 32;
             const int wt = wm ? __ffs(wm) - 1 : 32;
             if (wt < p) {  // a needed predecessor is still Waiting: re-poll the empty slots
+#ifdef CSZP2_TRACE
+                if (lane == 0 && g_trace) g_trace[t * 8 + 5]++;
+#endif
                 __nanosleep(32);
 #pragma unroll
                 for (int u = 0; u < LB_PER_LANE; u++)
@@ -265,6 +289,9 @@ __device__ __forceinline__ uint64_t lookback_finish(uint64_t *index, uint64_t t,
             break;
         }
         if (!done) {
+#ifdef CSZP2_TRACE
+            if (lane == 0 && g_trace) g_trace[t * 8 + 6]++;
+#endif
             j -= 32 * LB_PER_LANE;
             lookback_issue(index, j, w);
         }
@@ -272,6 +299,14 @@ __device__ __forceinline__ uint64_t lookback_finish(uint64_t *index, uint64_t t,
     if (lane == 0) st_relaxed_u64(&index[t], FLAG_P | rbits | (excl + agg));
     *range_out = rbits != 0;
     return excl;
+}
+
+// Issue the first window and resolve (used by the compression consumer warp).
+__device__ __forceinline__ uint64_t lookback(uint64_t *index, uint64_t t, uint64_t agg, bool bad,
+                                             bool *range_out) {
+    LookbackWindow w;
+    lookback_issue(index, static_cast<int64_t>(t) - 1, w);
+    return lookback_finish(index, t, agg, bad, w, range_out);
 }
 
 // ------------------------------------------------------------------ REL: min/max
@@ -395,10 +430,25 @@ struct HdrStatic {
     double eb_user;    // header bytes 24..31
 };
 
-// Three rotating tile buffers per CTA: tile i is encoded out of one (and its
-// payload staged back into it), tile i-1's staged payload waits in another for its
-// prefix, and tile i+1 streams into the third.
+// Warp-specialised compression CTA (NT_COMP = 384 threads):
+//   producers  warps 0-7  one thread per 32-value block; claim a tile from the
+//                         atomic ticket, TMA-load it, encode it (❶ ❷), publish its
+//                         aggregate, stage its payload in the tile's own buffer;
+//   resolvers  warps 8-9  decoupled lookback (❸) of each staged tile (round-robin);
+//   writers    warps 10-11 copy each resolved tile's payload to its place (❹).
+// NBUF tile buffers rotate through full -> staged -> resolved -> empty mbarriers.
+// A producer claims a tile only after it owns an empty buffer, and nothing it does
+// afterwards waits on a lookback, so every claimed tile's aggregate appears within
+// one load + encode: no tile is ever held behind a lookback wait (that coupling
+// serialised the whole machine on the P frontier in earlier versions).
 constexpr int NBUF = 3;
+constexpr int NT_COMP = NT + 128;
+constexpr int RESOLVE_WARP = NT / 32;          // warps 8, 9
+constexpr int NRESOLVE = 2;                    // resolver warps (tiles round-robin)
+constexpr int WRITER0 = NT + 32 * NRESOLVE;    // first writer thread
+constexpr int NWRITER = NT_COMP - WRITER0;     // 64 writer threads
+constexpr uint32_t BAR_PROD = 1, BAR_WRITE = 2;
+
 template <typename T>
 struct CompLayout {
     static constexpr uint32_t STRIDE = Traits<T>::TILE_BYTES + (sizeof(T) == 4 ? 1024 : 0);
@@ -410,11 +460,11 @@ constexpr int compress_smem_bytes() {
 }
 
 // Copy a tile's staged payload (smem, tile-relative, 16-byte aligned base) to its
-// global byte range [dst0, dst0 + bytes): 16-byte aligned chunks by coalesced
-// 128-bit stores (funnel-shifted out of smem), the unaligned head/tail by bytes.
+// global byte range [dst0, dst0 + bytes) with threads w = 0..nw-1: 16-byte aligned
+// chunks by coalesced 128-bit stores (funnel-shifted out of smem), the unaligned
+// head/tail by bytes.
 __device__ __forceinline__ void write_payload(const uint8_t *stg, uint8_t *out, uint64_t dst0,
-                                              uint32_t bytes) {
-    const int tid = threadIdx.x;
+                                              uint32_t bytes, int w, int nw) {
     const uint64_t dst1 = dst0 + bytes;
     const uint64_t a0 = roundup16(dst0), a1 = dst1 & ~uint64_t(15);
     if (a0 < a1) {
@@ -422,9 +472,9 @@ __device__ __forceinline__ void write_payload(const uint8_t *stg, uint8_t *out, 
         const uint32_t sh = 8u * (s0 & 3u);
         const uint32_t *sw = reinterpret_cast<const uint32_t *>(stg) + (s0 >> 2);
         const uint32_t nchunks = static_cast<uint32_t>((a1 - a0) >> 4);
-        for (uint32_t c = tid; c < nchunks; c += NT) {
-            const uint32_t *w = sw + 4 * c;
-            const uint32_t v0 = w[0], v1 = w[1], v2 = w[2], v3 = w[3], v4 = w[4];
+        for (uint32_t c = w; c < nchunks; c += nw) {
+            const uint32_t *p = sw + 4 * c;
+            const uint32_t v0 = p[0], v1 = p[1], v2 = p[2], v3 = p[3], v4 = p[4];
             uint4 o;
             o.x = __funnelshift_r(v0, v1, sh);
             o.y = __funnelshift_r(v1, v2, sh);
@@ -432,28 +482,21 @@ __device__ __forceinline__ void write_payload(const uint8_t *stg, uint8_t *out, 
             o.w = __funnelshift_r(v3, v4, sh);
             *reinterpret_cast<uint4 *>(out + a0 + 16ull * c) = o;
         }
-        if (tid >= NT - 32 && tid < NT - 16) {  // head bytes
-            const uint64_t o = dst0 + (tid - (NT - 32));
+        if (w < 16) {  // head bytes
+            const uint64_t o = dst0 + w;
             if (o < a0) out[o] = stg[o - dst0];
-        } else if (tid >= NT - 16) {  // tail bytes
-            const uint64_t o = a1 + (tid - (NT - 16));
+        } else if (w < 32) {  // tail bytes
+            const uint64_t o = a1 + (w - 16);
             if (o < dst1) out[o] = stg[o - dst0];
         }
-    } else if (tid >= NT - 32) {  // the whole payload is < 32 bytes
-        const uint64_t o = dst0 + (tid - (NT - 32));
+    } else if (w < 32) {  // the whole payload is < 32 bytes
+        const uint64_t o = dst0 + w;
         if (o < dst1) out[o] = stg[o - dst0];
     }
 }
 
-// Persistent compression kernel. Tiles are claimed in order from an atomic
-// ticket (every predecessor a lookback waits for belongs to a running CTA) and
-// loaded by TMA one tile ahead. Iteration i: encode tile i (❶ ❷, payload staged in
-// smem at tile-relative offsets), publish its aggregate, claim + prefetch tile
-// i+1, then resolve the prefix of tile i-1 (❸) — by now usually one L2 round trip —
-// and write tile i-1 out (❹). A claimed tile is never held behind a lookback wait,
-// which would serialise the whole machine on the P frontier.
 template <typename T, bool OUTLIER>
-__global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) compress_kernel(
+__global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kernel(
     const __grid_constant__ CUtensorMap tmap, const T *__restrict__ in, const Geom g,
     const double eb_abs_arg, const int eb_from_header, uint8_t *__restrict__ out,
     unsigned *__restrict__ ticket, uint64_t *__restrict__ d_out_bytes, const HdrStatic hs) {
@@ -461,23 +504,25 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) compress_kernel(
     constexpr uint32_t STRIDE = CompLayout<T>::STRIDE;
     uint8_t *bufs = reinterpret_cast<uint8_t *>(
         (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    __shared__ uint64_t s_bar[NBUF];
-    __shared__ uint32_t s_tk[NBUF];
+    __shared__ uint64_t s_full[NBUF], s_staged[NBUF], s_resolved[NBUF], s_empty[NBUF];
+    __shared__ uint32_t s_tk[NBUF], s_agg[NBUF];
+    __shared__ uint64_t s_excl[NBUF];
+    __shared__ uint8_t s_bad[NBUF], s_rng[NBUF];
     __shared__ uint32_t s_warp[NT / 32];
-    __shared__ uint64_t s_excl;
-    __shared__ bool s_rng;
+    __shared__ volatile uint32_t s_end;  // producers' final iteration (end marker)
 
     const int tid = threadIdx.x;
+    const int warp = tid >> 5;
     const uint64_t T_eff = g.T ? g.T : 1;
     uint64_t *index = reinterpret_cast<uint64_t *>(out + 64);
 
-    // TMA thread: start the load of tile `tk` into buffer `bi` (always arrives on
-    // the buffer's mbarrier so its phase advances even without data)
+    // producer leader: start the load of tile `tk` into buffer `bi` (always arrives
+    // on the buffer's full barrier so its phase advances even without data)
     auto issue = [&](uint64_t tk, int bi) {
-        uint64_t *bar = &s_bar[bi];
+        uint64_t *bar = &s_full[bi];
         uint8_t *dst = bufs + bi * STRIDE;
         const uint64_t b0 = tk * BPT;
-        if (tk < T_eff && b0 < g.nfull) {
+        if (b0 < g.nfull) {
             if (Traits<T>::ROWS == 1) {
                 mbar_expect_tx(bar, BPT * 128);
                 tma_load_2d(dst, &tmap, 0, static_cast<int>(b0), bar);
@@ -491,45 +536,59 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) compress_kernel(
             mbar_expect_tx(bar, 0);
         }
     };
-
-    if (tid == TMA_TID) {
-        for (int i = 0; i < NBUF; i++) mbar_init(&s_bar[i], 1);
-        fence_mbar_init();
+    auto claim = [&](int bi) {
         const uint32_t tk = atomicAdd(ticket, 1u);
-        s_tk[0] = tk;
-        issue(tk, 0);
+        if (tk < T_eff) TRACE(tk, 0, gtimer());
+        s_tk[bi] = tk;
+        if (tk < T_eff) issue(tk, bi);
+    };
+
+    if (tid == 0) {
+        s_end = 0xFFFFFFFFu;
+        for (int i = 0; i < NBUF; i++) {
+            mbar_init(&s_full[i], 1);
+            mbar_init(&s_staged[i], 1);
+            mbar_init(&s_resolved[i], 1);
+            mbar_init(&s_empty[i], 1);
+        }
+        fence_mbar_init();
+        claim(0);
     }
     __syncthreads();
 
-    // constants of the arithmetic contract (FORMAT.md §6.2)
-    const double eb_abs =
-        eb_from_header ? *reinterpret_cast<const volatile double *>(out + 32) : eb_abs_arg;
-    const auto K = make_consts(eb_abs, static_cast<T *>(nullptr));
-
-    uint64_t prev_t = ~uint64_t(0);  // tile encoded in the previous iteration (uniform)
-    uint32_t prev_agg = 0;
-    bool prev_bad = false;
-    LookbackWindow win;
-    for (uint32_t it = 0;; ++it) {
-        const int cur = it % NBUF;
-        const uint64_t t = s_tk[cur];
-        const bool have_cur = t < T_eff;
-        const bool have_prev = prev_t != ~uint64_t(0);
-        if (!have_cur && !have_prev) break;
-        const bool do_lookback = have_prev && g.T && prev_t > 0;
-        if (do_lookback && tid < 32)  // predecessors' descriptors fly while this tile encodes
-            lookback_issue(index, static_cast<int64_t>(prev_t) - 1, win);
-
-        uint32_t agg = 0;
-        bool any_bad = false;
-        if (have_cur) {
-            uint8_t *tile = bufs + cur * STRIDE;
+    if (warp < RESOLVE_WARP) {
+        // ============================== producers
+        const double eb_abs =
+            eb_from_header ? *reinterpret_cast<const volatile double *>(out + 32) : eb_abs_arg;
+        const auto K = make_consts(eb_abs, static_cast<T *>(nullptr));
+        for (uint32_t it = 0;; ++it) {
+            const int k = it % NBUF;
+            named_sync(BAR_PROD, NT);  // s_tk[k] (claimed by thread 0) visible
+            const uint64_t t = s_tk[k];
+            if (t >= T_eff) {
+                if (tid == 0) {  // end marker: release every resolver's pending wait
+                    s_end = it;
+                    for (int j = 0; j < NRESOLVE; j++) mbar_arrive(&s_staged[(it + j) % NBUF]);
+                }
+                break;
+            }
+            // Prefetch: claim the next tile now if its buffer is already free (the
+            // claimed tile is then held only through this tile's encode, never
+            // through a lookback); otherwise claim after publishing (below).
+            const uint32_t in_ = it + 1;
+            const int k2 = in_ % NBUF;
+            bool claimed = false;
+            if (tid == 0 && (in_ < NBUF || mbar_try_wait(&s_empty[k2], (in_ / NBUF - 1) & 1))) {
+                claim(k2);
+                claimed = true;
+            }
+            uint8_t *tile = bufs + k * STRIDE;
             const uint64_t b = t * BPT + tid;
             const bool active = b < g.nb;
             const bool full = b < g.nfull;
-            mbar_wait(&s_bar[cur], (it / NBUF) & 1);
+            mbar_wait(&s_full[k], (it / NBUF) & 1);
+            if (tid == 0) TRACE(t, 1, gtimer());
 
-            // ---- load the block's 32 values
             T x[L];
             uint32_t valid = L;
             if (full) {
@@ -540,7 +599,7 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) compress_kernel(
                 for (int i = 0; i < L; i++) x[i] = (i < (int)valid) ? in[b * L + i] : T(0);
             }
 
-            // ---- ❶ pre-quantization + in-block first-order difference
+            // ❶ pre-quantization + in-block first-order difference
             bool bad = false;
             int q[L];
 #pragma unroll
@@ -553,14 +612,14 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) compress_kernel(
             uint32_t a[L];
             uint32_t sign = 0, or_rest = 0;
 #pragma unroll
-            for (int i = 0; i < L; i++) {
+            for (int i = L - 1; i >= 0; i--) {
                 const int d = q[i] - (i ? q[i - 1] : 0);
                 a[i] = static_cast<uint32_t>(d < 0 ? -d : d);
-                sign |= static_cast<uint32_t>(d < 0) << i;
+                sign = __funnelshift_l(static_cast<uint32_t>(d), sign, 1);  // bit i = d_i < 0
                 if (i) or_rest |= a[i];
             }
 
-            // ---- ❷ fixed lengths and the fine-tuned Plain/Outlier selection
+            // ❷ fixed lengths and the fine-tuned Plain/Outlier selection
             const int fl_p = 32 - __clz(or_rest | a[0]);
             uint32_t size = fl_p ? 4u * (1u + fl_p) : 0u;
             uint32_t obyte = static_cast<uint32_t>(fl_p);
@@ -582,19 +641,21 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) compress_kernel(
             }
             if (!K.ok) bad = true;
 
-            // ---- intra-tile scan ("Reduce"); every thread is done reading `tile` after it
-            any_bad = __syncthreads_or(bad);
-            const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg);
-            if (tid == 0 && g.T) publish_aggregate(index, t, agg, any_bad);
-            if (tid == TMA_TID) {  // claim + prefetch the next tile right behind the publish
-                const int nxt = (it + 1) % NBUF;
-                const uint32_t tn = atomicAdd(ticket, 1u);
-                s_tk[nxt] = tn;
-                if (tn < T_eff) issue(tn, nxt);
+            // intra-tile scan ("Reduce"); the producers are done reading `tile` after it
+            const bool any_bad = named_sync_or(BAR_PROD, NT, bad);
+            uint32_t agg;
+            const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg, BAR_PROD);
+            if (tid == 0) {
+                if (g.T) publish_aggregate(index, t, agg, any_bad);
+                TRACE(t, 2, gtimer());
+                if (!claimed) {  // nothing unpublished is held while waiting here
+                    if (in_ >= NBUF) mbar_wait(&s_empty[k2], (in_ / NBUF - 1) & 1);
+                    claim(k2);
+                }
             }
             if (active) out[g.O + b] = static_cast<uint8_t>(obyte);  // ❹ offset bytes
 
-            // ---- ❷ payload staged at its tile-relative byte offset
+            // ❷ payload staged at its tile-relative byte offset
             if (size) {
                 uint8_t *p = tile + my_excl;
                 st_u32_unaligned(p, sign);
@@ -608,45 +669,74 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) compress_kernel(
                     const int sh = 32 - fl;
 #pragma unroll
                     for (int i = 0; i < L; i++) a[i] <<= sh;
-                    for (int k = fl - 1; k >= 0; k--) {  // planes top-down, 2 ops per bit
+                    for (int kk = fl - 1; kk >= 0; kk--) {  // planes top-down, 2 ops per bit
                         uint32_t w = 0;
 #pragma unroll
                         for (int i = L - 1; i >= 0; i--) shift_bit_into(a[i], w);
-                        st_u32_unaligned(p + 4 * k, w);
+                        st_u32_unaligned(p + 4 * kk, w);
                     }
                 }
             }
-        }
-
-        if (have_prev) {
-            // ---- ❸ prefix of the previous tile, then ❹ its payload to global
-            if (tid < 32) {
-                bool rng = prev_bad;
-                const uint64_t e =
-                    do_lookback ? lookback_finish(index, prev_t, prev_agg, prev_bad, win, &rng) : 0;
-                if (tid == 0) {
-                    s_excl = e;
-                    s_rng = rng;
-                }
+            named_sync(BAR_PROD, NT);  // staging complete
+            if (tid == 0) {
+                s_agg[k] = agg;
+                s_bad[k] = any_bad;
+                TRACE(t, 4, gtimer());
+                mbar_arrive(&s_staged[k]);
             }
-            __syncthreads();
-            const uint64_t excl = s_excl;
-            const uint8_t *stg = bufs + ((it + NBUF - 1) % NBUF) * STRIDE;
+        }
+    } else if (warp < RESOLVE_WARP + NRESOLVE) {
+        // ============================== resolvers: ❸, tile i by warp i % NRESOLVE.
+        // Lookbacks are independent (a resolver may walk past a neighbour's A that
+        // has not become P yet), so two in flight halve the per-tile latency.
+        const int lane = tid & 31;
+        for (uint32_t it = warp - RESOLVE_WARP;; it += NRESOLVE) {
+            const int k = it % NBUF;
+            mbar_wait(&s_staged[k], (it / NBUF) & 1);
+            if (it >= s_end) {
+                if (lane == 0 && it == s_end) mbar_arrive(&s_resolved[k]);  // writers' end
+                break;
+            }
+            const uint64_t t = s_tk[k];
+            const uint32_t agg = s_agg[k];
+            const bool bad = s_bad[k];
+            bool rng = bad;
+            const uint64_t e = (g.T && t > 0) ? lookback(index, t, agg, bad, &rng) : 0;
+            if (lane == 0) {
+                s_excl[k] = e;
+                s_rng[k] = rng;
+                TRACE(t, 3, gtimer());
+                mbar_arrive(&s_resolved[k]);
+            }
+        }
+    } else {
+        // ============================== writers: ❹ payload, pads, header
+        const int w = tid - WRITER0;
+        const double eb_abs =
+            eb_from_header ? *reinterpret_cast<const volatile double *>(out + 32) : eb_abs_arg;
+        for (uint32_t it = 0;; ++it) {
+            const int k = it % NBUF;
+            mbar_wait(&s_resolved[k], (it / NBUF) & 1);
+            if (it >= s_end) break;
+            const uint64_t t = s_tk[k];
+            const uint64_t excl = s_excl[k];
+            const uint32_t agg = s_agg[k];
             const uint64_t dst0 = g.D + excl;
-            write_payload(stg, out, dst0, prev_agg);
-            if (prev_t == T_eff - 1) {  // last tile: pads, header, d_out_bytes
-                const uint64_t dst1 = dst0 + prev_agg;
-                if (tid >= 32 && tid < 48) {  // zero pad after the payload
-                    const uint64_t o = dst1 + (tid - 32);
+            write_payload(bufs + k * STRIDE, out, dst0, agg, w, NWRITER);
+            if (t == T_eff - 1) {  // last tile: pads, header, d_out_bytes
+                const uint64_t dst1 = dst0 + agg;
+                if (w >= 32 && w < 48) {  // zero pad after the payload
+                    const uint64_t o = dst1 + (w - 32);
                     if (o < roundup16(dst1)) out[o] = 0;
                 }
-                if (tid >= 64 && tid < 80) {  // zero pad after the offset bytes
-                    const uint64_t o = g.O + g.nb + (tid - 64);
+                static_assert(NWRITER >= 64, "pads use writer threads 32..63");
+                if (w >= 48 && w < 64) {  // zero pad after the offset bytes
+                    const uint64_t o = g.O + g.nb + (w - 48);
                     if (o < g.D) out[o] = 0;
                 }
-                if (tid == 0) {
-                    const uint32_t status = s_rng ? ST_RANGE : 0u;
-                    const uint64_t pb = status ? 0 : excl + prev_agg;
+                if (w == 0) {
+                    const uint32_t status = s_rng[k] ? ST_RANGE : 0u;
+                    const uint64_t pb = status ? 0 : excl + agg;
                     const uint64_t total = roundup16(g.D + pb);
                     uint64_t *h = reinterpret_cast<uint64_t *>(out);
                     h[0] = MAGIC | (static_cast<uint64_t>(hs.word1) << 32);
@@ -660,12 +750,9 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) compress_kernel(
                     if (d_out_bytes) *d_out_bytes = total;
                 }
             }
+            named_sync(BAR_WRITE, NWRITER);  // all writers done reading buffer k
+            if (w == 0) mbar_arrive(&s_empty[k]);
         }
-        if (!have_cur) break;  // the previous tile was the last one this CTA held
-        prev_t = t;
-        prev_agg = agg;
-        prev_bad = any_bad;
-        __syncthreads();  // staging reads done before the buffer is refilled; s_tk visible
     }
 }
 

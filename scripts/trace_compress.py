@@ -1,0 +1,43 @@
+"""Per-tile timeline of the compression kernel (debug build libcszp2_trace.so)."""
+import sys, os, ctypes
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np, torch
+from synthetic import CONFIGS, make_field
+lib = ctypes.CDLL(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "paper_conf_sc_huangdlc24_b200", "libcszp2_trace.so"))
+vp, u64, i32, dbl = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int, ctypes.c_double
+lib.cszp2_compress.argtypes = [vp, u64, i32, dbl, i32, i32, vp, vp, vp]
+lib.cszp2_compress_bound.argtypes = [u64, i32]; lib.cszp2_compress_bound.restype = u64
+lib.cszp2_debug_set_trace.argtypes = [vp]
+for cfg in sys.argv[1:]:
+    spec = CONFIGS[cfg]
+    x = make_field(cfg, "cuda"); n = x.numel()
+    T = -(-(-(-n // 32)) // 256)
+    out = torch.empty(lib.cszp2_compress_bound(n, 0), dtype=torch.uint8, device="cuda")
+    tr = torch.zeros(T * 8, dtype=torch.int64, device="cuda")
+    lib.cszp2_debug_set_trace(ctypes.c_void_p(tr.data_ptr()))
+    st = torch.cuda.current_stream().cuda_stream
+    for rep in range(3):
+        tr.zero_()
+        lib.cszp2_compress(ctypes.c_void_p(x.data_ptr()), n, 0, spec.ebs[-1], 1, 1, ctypes.c_void_p(out.data_ptr()), None, ctypes.c_void_p(st))
+        torch.cuda.synchronize()
+    a = tr.view(T, 8).cpu().numpy().astype(np.int64)
+    t0 = a[:, 0][a[:, 0] > 0].min()
+    a[:, :5] -= t0
+    claim, data, pub, res, staged, polls, moves = [a[:, i] for i in range(7)]
+    print(f"== {cfg}: T={T} span={(res.max())/1e3:.1f}us rate={T/(res.max()/1e3):.1f} tiles/us")
+    def q(v): return " ".join(f"{np.percentile(v,p):7.2f}" for p in (5,25,50,75,95,99))
+    print("pct                5      25      50      75      95      99  (us)")
+    print("claim->data   ", q((data-claim)/1e3))
+    print("data->pubA    ", q((pub-data)/1e3))
+    print("pubA->staged  ", q((staged-pub)/1e3))
+    print("pubA->resolved", q((res[1:]-pub[1:])/1e3))
+    print("claim->resolved", q((res[1:]-claim[1:])/1e3))
+    print("polls mean", polls.mean(), "max", polls.max(), "moves mean", moves.mean())
+    # frontier: resolved time vs tile index; claim order vs time
+    order = np.argsort(claim)
+    print("claims per us (median over 10us windows):", np.median(np.diff(np.searchsorted(np.sort(claim), np.arange(0, claim.max(), 10000))))/10)
+    # lag between claim of tile t and resolve of tile t: grows?
+    for frac in (0.1, 0.3, 0.5, 0.7, 0.9):
+        i = int(frac * T); sl = slice(i, i + 200)
+        print(f" tiles@{frac:.1f}: claim->res {np.median(res[sl]-claim[sl])/1e3:7.2f}us  claim-gap to prev tile claim {np.median(np.diff(claim[sl]))/1e3:6.3f}us  polls {polls[sl].mean():.2f}")
+    del x, out, tr; torch.cuda.empty_cache()
