@@ -539,6 +539,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
     auto claim = [&](int bi) {
         const uint32_t tk = atomicAdd(ticket, 1u);
         if (tk < T_eff) TRACE(tk, 0, gtimer());
+        if (tk < T_eff) TRACE(tk, 7, blockIdx.x);
         s_tk[bi] = tk;
         if (tk < T_eff) issue(tk, bi);
     };

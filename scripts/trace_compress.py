@@ -41,3 +41,17 @@ for cfg in sys.argv[1:]:
         i = int(frac * T); sl = slice(i, i + 200)
         print(f" tiles@{frac:.1f}: claim->res {np.median(res[sl]-claim[sl])/1e3:7.2f}us  claim-gap to prev tile claim {np.median(np.diff(claim[sl]))/1e3:6.3f}us  polls {polls[sl].mean():.2f}")
     del x, out, tr; torch.cuda.empty_cache()
+    # per-CTA timelines (slot 7 = CTA id)
+    cta = a[:, 7]
+    per = []
+    waits = []; comp = []; stg = []
+    for c in np.unique(cta)[:300]:
+        idx = np.where(cta == c)[0]
+        idx = idx[np.argsort(data[idx])]
+        if len(idx) < 3: continue
+        d, p_, s_ = data[idx], pub[idx], staged[idx]
+        per.append(np.median(np.diff(d)))
+        waits.append(np.median(d[1:] - s_[:-1])); comp.append(np.median(p_ - d)); stg.append(np.median(s_ - p_))
+    print(f"per-CTA period {np.median(per)/1e3:.2f}us  staged->next data {np.median(waits)/1e3:.2f}us  compute {np.median(comp)/1e3:.2f}us  staging {np.median(stg)/1e3:.2f}us")
+    w = np.array([x for x in waits])
+    print("staged->next data pct", q(w/1e3))
