@@ -289,9 +289,7 @@ __device__ __forceinline__ uint64_t lookback_finish(uint64_t *index, uint64_t t,
             break;
         }
         if (!done) {
-#ifdef CSZP2_TRACE
-            if (lane == 0 && g_trace) g_trace[t * 8 + 6]++;
-#endif
+
             j -= 32 * LB_PER_LANE;
             lookback_issue(index, j, w);
         }
@@ -430,39 +428,46 @@ struct HdrStatic {
     double eb_user;    // header bytes 24..31
 };
 
-// Warp-specialised compression CTA (NT_COMP = 384 threads):
-//   producers  warps 0-7  one thread per 32-value block; claim a tile from the
-//                         atomic ticket, TMA-load it, encode it (❶ ❷), publish its
-//                         aggregate, stage its payload in the tile's own buffer;
-//   resolvers  warps 8-9  decoupled lookback (❸) of each staged tile (round-robin);
-//   writers    warps 10-11 copy each resolved tile's payload to its place (❹).
-// NBUF tile buffers rotate through full -> staged -> resolved -> empty mbarriers.
-// A producer claims a tile only after it owns an empty buffer, and nothing it does
-// afterwards waits on a lookback, so every claimed tile's aggregate appears within
-// one load + encode: no tile is ever held behind a lookback wait (that coupling
-// serialised the whole machine on the P frontier in earlier versions).
-constexpr int NBUF = 3;
+// Warp-specialised compression CTA (NT_COMP = 384 threads = 12 warps):
+//   producers  warps 0-7   one thread per 32-value block: take a loaded tile, read it
+//                          into registers (freeing its TMA buffer at once), encode it
+//                          (❶ ❷), publish its aggregate, stage its payload in a
+//                          byte ring, queue it;
+//   loader     warp 8      claims tiles from the atomic ticket and TMA-loads them into
+//                          two input buffers, one tile ahead of the producers;
+//   resolver   warp 9      decoupled lookback (❸) of the queued tiles, in order (a
+//                          second resolver warp starts lookbacks before their
+//                          predecessors are published and measured slower);
+//   writers    warps 10-11 copy each resolved payload out of the ring to its place
+//                          (❹), in order, then free its ring bytes and queue slot.
+// Input buffers are released as soon as the producers hold the values, and the
+// (small, at useful compression ratios) payloads wait for their prefix in the ring,
+// so neither the loads nor the producers ever wait behind a lookback: a claimed
+// tile's aggregate appears within one load + encode of the claim.
 constexpr int NT_COMP = NT + 128;
-constexpr int RESOLVE_WARP = NT / 32;          // warps 8, 9
-constexpr int NRESOLVE = 2;                    // resolver warps (tiles round-robin)
-constexpr int WRITER0 = NT + 32 * NRESOLVE;    // first writer thread
-constexpr int NWRITER = NT_COMP - WRITER0;     // 64 writer threads
+constexpr int LOADER_WARP = NT / 32;       // warp 8
+constexpr int RESOLVE_WARP = NT / 32 + 1;  // warps 9-10
+constexpr int NRESOLVE = 1;                // lookback warps (queue entries round-robin)
+constexpr int WRITER0 = NT + 64;           // first writer thread (warps 10-11)
+constexpr int NWRITER = NT_COMP - WRITER0; // 64 writer threads
+constexpr int NQ = 16;                     // queue slots (tiles staged ahead of the writers)
 constexpr uint32_t BAR_PROD = 1, BAR_WRITE = 2;
 
 template <typename T>
 struct CompLayout {
-    static constexpr uint32_t STRIDE = Traits<T>::TILE_BYTES + (sizeof(T) == 4 ? 1024 : 0);
-    static constexpr int SMEM = NBUF * STRIDE + 1024;
+    static constexpr uint32_t IN_BYTES = Traits<T>::TILE_BYTES;  // one TMA tile
+    static constexpr uint32_t RING = sizeof(T) == 4 ? 40960u : 36864u;  // >= one max payload
+    static constexpr int SMEM = 2 * IN_BYTES + RING + 64 + 1024;
 };
 template <typename T>
 constexpr int compress_smem_bytes() {
     return CompLayout<T>::SMEM;
 }
 
-// Copy a tile's staged payload (smem, tile-relative, 16-byte aligned base) to its
-// global byte range [dst0, dst0 + bytes) with threads w = 0..nw-1: 16-byte aligned
-// chunks by coalesced 128-bit stores (funnel-shifted out of smem), the unaligned
-// head/tail by bytes.
+// Copy a tile's staged payload (smem, 16-byte aligned base) to its global byte
+// range [dst0, dst0 + bytes) with threads w = 0..nw-1: 16-byte aligned chunks by
+// coalesced 128-bit stores (funnel-shifted out of smem), the unaligned head/tail by
+// bytes.
 __device__ __forceinline__ void write_payload(const uint8_t *stg, uint8_t *out, uint64_t dst0,
                                               uint32_t bytes, int w, int nw) {
     const uint64_t dst1 = dst0 + bytes;
@@ -500,95 +505,70 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
     const __grid_constant__ CUtensorMap tmap, const T *__restrict__ in, const Geom g,
     const double eb_abs_arg, const int eb_from_header, uint8_t *__restrict__ out,
     unsigned *__restrict__ ticket, uint64_t *__restrict__ d_out_bytes, const HdrStatic hs) {
+    using LY = CompLayout<T>;
     extern __shared__ uint8_t smem_raw[];
-    constexpr uint32_t STRIDE = CompLayout<T>::STRIDE;
-    uint8_t *bufs = reinterpret_cast<uint8_t *>(
+    uint8_t *inbuf = reinterpret_cast<uint8_t *>(
         (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    __shared__ uint64_t s_full[NBUF], s_staged[NBUF], s_resolved[NBUF], s_empty[NBUF];
-    __shared__ uint32_t s_tk[NBUF], s_agg[NBUF];
-    __shared__ uint64_t s_excl[NBUF];
-    __shared__ uint8_t s_bad[NBUF], s_rng[NBUF];
+    uint8_t *ring = inbuf + 2 * LY::IN_BYTES;
+    __shared__ uint64_t s_full[2], s_free[2];                      // input buffers
+    __shared__ uint64_t s_staged[NQ], s_resolved[NQ], s_done[NQ];  // queue slots
+    __shared__ uint32_t s_tkin[2];
+    __shared__ uint64_t s_qt[NQ], s_qexcl[NQ];
+    __shared__ uint32_t s_qagg[NQ], s_qpos[NQ];
+    __shared__ uint8_t s_qbad[NQ], s_qrng[NQ];
     __shared__ uint32_t s_warp[NT / 32];
-    __shared__ volatile uint32_t s_end;  // producers' final iteration (end marker)
+    __shared__ uint32_t s_pos;
+    __shared__ volatile uint32_t s_tail;  // ring bytes released by the writers
+    __shared__ volatile uint32_t s_end;   // queue index of the end marker
 
     const int tid = threadIdx.x;
     const int warp = tid >> 5;
     const uint64_t T_eff = g.T ? g.T : 1;
     uint64_t *index = reinterpret_cast<uint64_t *>(out + 64);
 
-    // producer leader: start the load of tile `tk` into buffer `bi` (always arrives
-    // on the buffer's full barrier so its phase advances even without data)
-    auto issue = [&](uint64_t tk, int bi) {
-        uint64_t *bar = &s_full[bi];
-        uint8_t *dst = bufs + bi * STRIDE;
-        const uint64_t b0 = tk * BPT;
-        if (b0 < g.nfull) {
-            if (Traits<T>::ROWS == 1) {
-                mbar_expect_tx(bar, BPT * 128);
-                tma_load_2d(dst, &tmap, 0, static_cast<int>(b0), bar);
-            } else {
-                const bool second = (b0 + BPT / 2) < g.nfull;
-                mbar_expect_tx(bar, second ? 2 * BPT * 128 : BPT * 128);
-                tma_load_2d(dst, &tmap, 0, static_cast<int>(2 * b0), bar);
-                if (second) tma_load_2d(dst + BPT * 128, &tmap, 0, static_cast<int>(2 * b0 + BPT), bar);
-            }
-        } else {
-            mbar_expect_tx(bar, 0);
-        }
-    };
-    auto claim = [&](int bi) {
-        const uint32_t tk = atomicAdd(ticket, 1u);
-        if (tk < T_eff) TRACE(tk, 0, gtimer());
-        if (tk < T_eff) TRACE(tk, 7, blockIdx.x);
-        s_tk[bi] = tk;
-        if (tk < T_eff) issue(tk, bi);
-    };
-
     if (tid == 0) {
         s_end = 0xFFFFFFFFu;
-        for (int i = 0; i < NBUF; i++) {
+        s_tail = 0;
+        for (int i = 0; i < 2; i++) {
             mbar_init(&s_full[i], 1);
+            mbar_init(&s_free[i], 1);
+        }
+        for (int i = 0; i < NQ; i++) {
             mbar_init(&s_staged[i], 1);
             mbar_init(&s_resolved[i], 1);
-            mbar_init(&s_empty[i], 1);
+            mbar_init(&s_done[i], 1);
         }
         fence_mbar_init();
-        claim(0);
     }
     __syncthreads();
 
-    if (warp < RESOLVE_WARP) {
+    if (warp < LOADER_WARP) {
         // ============================== producers
         const double eb_abs =
             eb_from_header ? *reinterpret_cast<const volatile double *>(out + 32) : eb_abs_arg;
         const auto K = make_consts(eb_abs, static_cast<T *>(nullptr));
+        uint32_t head = 0;  // ring allocation cursor (thread 0)
         for (uint32_t it = 0;; ++it) {
-            const int k = it % NBUF;
-            named_sync(BAR_PROD, NT);  // s_tk[k] (claimed by thread 0) visible
-            const uint64_t t = s_tk[k];
-            if (t >= T_eff) {
-                if (tid == 0) {  // end marker: release every resolver's pending wait
+            const int bi = it & 1;
+            const int q = it % NQ;
+            mbar_wait(&s_full[bi], (it >> 1) & 1);
+            const uint64_t t = s_tkin[bi];
+            if (t >= T_eff) {  // end marker for the resolver and the writers
+                if (tid == 0) {
+                    for (int j = 0; j < NRESOLVE; j++) {  // release every resolver's pending wait
+                        const uint32_t ij = it + j;
+                        if (ij >= NQ) mbar_wait(&s_done[ij % NQ], (ij / NQ - 1) & 1);
+                    }
                     s_end = it;
-                    for (int j = 0; j < NRESOLVE; j++) mbar_arrive(&s_staged[(it + j) % NBUF]);
+                    for (int j = 0; j < NRESOLVE; j++) mbar_arrive(&s_staged[(it + j) % NQ]);
                 }
                 break;
             }
-            // Prefetch: claim the next tile now if its buffer is already free (the
-            // claimed tile is then held only through this tile's encode, never
-            // through a lookback); otherwise claim after publishing (below).
-            const uint32_t in_ = it + 1;
-            const int k2 = in_ % NBUF;
-            bool claimed = false;
-            if (tid == 0 && (in_ < NBUF || mbar_try_wait(&s_empty[k2], (in_ / NBUF - 1) & 1))) {
-                claim(k2);
-                claimed = true;
-            }
-            uint8_t *tile = bufs + k * STRIDE;
+            if (tid == 0) TRACE(t, 1, gtimer());
+            const uint8_t *tile = inbuf + bi * LY::IN_BYTES;
             const uint64_t b = t * BPT + tid;
             const bool active = b < g.nb;
             const bool full = b < g.nfull;
-            mbar_wait(&s_full[k], (it / NBUF) & 1);
-            if (tid == 0) TRACE(t, 1, gtimer());
 
             T x[L];
             uint32_t valid = L;
@@ -602,19 +582,19 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
 
             // ❶ pre-quantization + in-block first-order difference
             bool bad = false;
-            int q[L];
+            int qv[L];
 #pragma unroll
-            for (int i = 0; i < L; i++) q[i] = quantize(x[i], K.inv, bad);
+            for (int i = 0; i < L; i++) qv[i] = quantize(x[i], K.inv, bad);
             if (!full) {  // tail block: q_i = q_{i-1} past n (FORMAT.md §6.4)
 #pragma unroll
                 for (int i = 1; i < L; i++)
-                    if (i >= (int)valid) q[i] = q[i - 1];
+                    if (i >= (int)valid) qv[i] = qv[i - 1];
             }
             uint32_t a[L];
             uint32_t sign = 0, or_rest = 0;
 #pragma unroll
             for (int i = L - 1; i >= 0; i--) {
-                const int d = q[i] - (i ? q[i - 1] : 0);
+                const int d = qv[i] - (i ? qv[i - 1] : 0);
                 a[i] = static_cast<uint32_t>(d < 0 ? -d : d);
                 sign = __funnelshift_l(static_cast<uint32_t>(d), sign, 1);  // bit i = d_i < 0
                 if (i) or_rest |= a[i];
@@ -642,23 +622,32 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
             }
             if (!K.ok) bad = true;
 
-            // intra-tile scan ("Reduce"); the producers are done reading `tile` after it
+            // intra-tile scan ("Reduce"); the input buffer is free after it
             const bool any_bad = named_sync_or(BAR_PROD, NT, bad);
+            if (tid == 0) mbar_arrive(&s_free[bi]);
             uint32_t agg;
             const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg, BAR_PROD);
             if (tid == 0) {
                 if (g.T) publish_aggregate(index, t, agg, any_bad);
                 TRACE(t, 2, gtimer());
-                if (!claimed) {  // nothing unpublished is held while waiting here
-                    if (in_ >= NBUF) mbar_wait(&s_empty[k2], (in_ / NBUF - 1) & 1);
-                    claim(k2);
-                }
+                // ring space (16-aligned, contiguous) and a queue slot
+                uint32_t pos = (head + 15u) & ~15u;
+                if ((pos % LY::RING) + agg > LY::RING) pos = (pos / LY::RING + 1) * LY::RING;
+                while (pos + agg > s_tail + LY::RING) __nanosleep(64);
+                head = pos + agg;
+                if (it >= NQ) mbar_wait(&s_done[q], (it / NQ - 1) & 1);
+                s_pos = pos;
+                s_qt[q] = t;
+                s_qagg[q] = agg;
+                s_qbad[q] = any_bad;
+                s_qpos[q] = pos;
             }
             if (active) out[g.O + b] = static_cast<uint8_t>(obyte);  // ❹ offset bytes
+            named_sync(BAR_PROD, NT);  // s_pos visible
 
-            // ❷ payload staged at its tile-relative byte offset
+            // ❷ payload staged in the ring at its tile-relative byte offset
             if (size) {
-                uint8_t *p = tile + my_excl;
+                uint8_t *p = ring + (s_pos % LY::RING) + my_excl;
                 st_u32_unaligned(p, sign);
                 p += 4;
                 if (OUTLIER && nob) {
@@ -680,34 +669,64 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
             }
             named_sync(BAR_PROD, NT);  // staging complete
             if (tid == 0) {
-                s_agg[k] = agg;
-                s_bad[k] = any_bad;
                 TRACE(t, 4, gtimer());
-                mbar_arrive(&s_staged[k]);
+                mbar_arrive(&s_staged[q]);
+            }
+        }
+    } else if (warp == LOADER_WARP) {
+        // ============================== loader: claim + TMA one tile ahead
+        if ((tid & 31) == 0) {
+            for (uint32_t it = 0;; ++it) {
+                const int bi = it & 1;
+                if (it >= 2) mbar_wait(&s_free[bi], (it / 2 - 1) & 1);
+                const uint32_t tk = atomicAdd(ticket, 1u);
+                s_tkin[bi] = tk;
+                uint64_t *bar = &s_full[bi];
+                if (tk >= T_eff) {
+                    mbar_arrive(bar);  // producers see the end
+                    break;
+                }
+                TRACE(tk, 0, gtimer());
+                TRACE(tk, 7, blockIdx.x);
+                uint8_t *dst = inbuf + bi * LY::IN_BYTES;
+                const uint64_t b0 = static_cast<uint64_t>(tk) * BPT;
+                if (b0 < g.nfull) {
+                    if (Traits<T>::ROWS == 1) {
+                        mbar_expect_tx(bar, BPT * 128);
+                        tma_load_2d(dst, &tmap, 0, static_cast<int>(b0), bar);
+                    } else {
+                        const bool second = (b0 + BPT / 2) < g.nfull;
+                        mbar_expect_tx(bar, second ? 2 * BPT * 128 : BPT * 128);
+                        tma_load_2d(dst, &tmap, 0, static_cast<int>(2 * b0), bar);
+                        if (second)
+                            tma_load_2d(dst + BPT * 128, &tmap, 0, static_cast<int>(2 * b0 + BPT), bar);
+                    }
+                } else {
+                    mbar_expect_tx(bar, 0);
+                }
             }
         }
     } else if (warp < RESOLVE_WARP + NRESOLVE) {
-        // ============================== resolvers: ❸, tile i by warp i % NRESOLVE.
-        // Lookbacks are independent (a resolver may walk past a neighbour's A that
-        // has not become P yet), so two in flight halve the per-tile latency.
+        // ============================== resolvers: ❸, queue entry i by warp i % NRESOLVE
         const int lane = tid & 31;
         for (uint32_t it = warp - RESOLVE_WARP;; it += NRESOLVE) {
-            const int k = it % NBUF;
-            mbar_wait(&s_staged[k], (it / NBUF) & 1);
+            const int q = it % NQ;
+            mbar_wait(&s_staged[q], (it / NQ) & 1);
             if (it >= s_end) {
-                if (lane == 0 && it == s_end) mbar_arrive(&s_resolved[k]);  // writers' end
+                if (lane == 0 && it == s_end) mbar_arrive(&s_resolved[q]);  // writer's end
                 break;
             }
-            const uint64_t t = s_tk[k];
-            const uint32_t agg = s_agg[k];
-            const bool bad = s_bad[k];
+            const uint64_t t = s_qt[q];
+            const uint32_t agg = s_qagg[q];
+            const bool bad = s_qbad[q];
+            if (lane == 0) TRACE(t, 6, gtimer());
             bool rng = bad;
             const uint64_t e = (g.T && t > 0) ? lookback(index, t, agg, bad, &rng) : 0;
             if (lane == 0) {
-                s_excl[k] = e;
-                s_rng[k] = rng;
+                s_qexcl[q] = e;
+                s_qrng[q] = rng;
                 TRACE(t, 3, gtimer());
-                mbar_arrive(&s_resolved[k]);
+                mbar_arrive(&s_resolved[q]);
             }
         }
     } else {
@@ -716,14 +735,15 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
         const double eb_abs =
             eb_from_header ? *reinterpret_cast<const volatile double *>(out + 32) : eb_abs_arg;
         for (uint32_t it = 0;; ++it) {
-            const int k = it % NBUF;
-            mbar_wait(&s_resolved[k], (it / NBUF) & 1);
+            const int q = it % NQ;
+            mbar_wait(&s_resolved[q], (it / NQ) & 1);
             if (it >= s_end) break;
-            const uint64_t t = s_tk[k];
-            const uint64_t excl = s_excl[k];
-            const uint32_t agg = s_agg[k];
+            const uint64_t t = s_qt[q];
+            const uint64_t excl = s_qexcl[q];
+            const uint32_t agg = s_qagg[q];
+            const uint32_t pos = s_qpos[q];
             const uint64_t dst0 = g.D + excl;
-            write_payload(bufs + k * STRIDE, out, dst0, agg, w, NWRITER);
+            write_payload(ring + (pos % LY::RING), out, dst0, agg, w, NWRITER);
             if (t == T_eff - 1) {  // last tile: pads, header, d_out_bytes
                 const uint64_t dst1 = dst0 + agg;
                 if (w >= 32 && w < 48) {  // zero pad after the payload
@@ -736,7 +756,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
                     if (o < g.D) out[o] = 0;
                 }
                 if (w == 0) {
-                    const uint32_t status = s_rng[k] ? ST_RANGE : 0u;
+                    const uint32_t status = s_qrng[q] ? ST_RANGE : 0u;
                     const uint64_t pb = status ? 0 : excl + agg;
                     const uint64_t total = roundup16(g.D + pb);
                     uint64_t *h = reinterpret_cast<uint64_t *>(out);
@@ -751,8 +771,11 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
                     if (d_out_bytes) *d_out_bytes = total;
                 }
             }
-            named_sync(BAR_WRITE, NWRITER);  // all writers done reading buffer k
-            if (w == 0) mbar_arrive(&s_empty[k]);
+            named_sync(BAR_WRITE, NWRITER);  // all writers done reading these ring bytes
+            if (w == 0) {
+                s_tail = pos + agg;  // writers go in order, so the ring frees in order
+                mbar_arrive(&s_done[q]);
+            }
         }
     }
 }

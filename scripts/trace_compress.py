@@ -23,7 +23,9 @@ for cfg in sys.argv[1:]:
     a = tr.view(T, 8).cpu().numpy().astype(np.int64)
     t0 = a[:, 0][a[:, 0] > 0].min()
     a[:, :5] -= t0
-    claim, data, pub, res, staged, polls, moves = [a[:, i] for i in range(7)]
+    a[:, 6] -= t0
+    claim, data, pub, res, staged, polls, rstart = [a[:, i] for i in range(7)]
+    moves = np.zeros_like(polls)
     print(f"== {cfg}: T={T} span={(res.max())/1e3:.1f}us rate={T/(res.max()/1e3):.1f} tiles/us")
     def q(v): return " ".join(f"{np.percentile(v,p):7.2f}" for p in (5,25,50,75,95,99))
     print("pct                5      25      50      75      95      99  (us)")
@@ -31,6 +33,8 @@ for cfg in sys.argv[1:]:
     print("data->pubA    ", q((pub-data)/1e3))
     print("pubA->staged  ", q((staged-pub)/1e3))
     print("pubA->resolved", q((res[1:]-pub[1:])/1e3))
+    print("staged->rstart", q((rstart[1:]-staged[1:])/1e3))
+    print("rstart->resolved", q((res[1:]-rstart[1:])/1e3))
     print("claim->resolved", q((res[1:]-claim[1:])/1e3))
     print("polls mean", polls.mean(), "max", polls.max(), "moves mean", moves.mean())
     # frontier: resolved time vs tile index; claim order vs time
