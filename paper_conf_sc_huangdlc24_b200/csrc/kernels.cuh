@@ -519,6 +519,9 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
     __shared__ uint32_t s_warp[NT / 32];
     __shared__ uint32_t s_pos;
     __shared__ volatile uint32_t s_tail;  // ring bytes released by the writers
+    __shared__ volatile uint32_t s_head;  // ring bytes allocated by the producers
+    __shared__ volatile uint32_t s_last_agg;  // payload bytes of the latest tile
+    __shared__ volatile uint32_t s_alloc_it;  // producer iterations holding ring space
     __shared__ volatile uint32_t s_end;   // queue index of the end marker
 
     const int tid = threadIdx.x;
@@ -529,6 +532,9 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
     if (tid == 0) {
         s_end = 0xFFFFFFFFu;
         s_tail = 0;
+        s_head = 0;
+        s_last_agg = 0;
+        s_alloc_it = 0;
         for (int i = 0; i < 2; i++) {
             mbar_init(&s_full[i], 1);
             mbar_init(&s_free[i], 1);
@@ -635,6 +641,9 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
                 if ((pos % LY::RING) + agg > LY::RING) pos = (pos / LY::RING + 1) * LY::RING;
                 while (pos + agg > s_tail + LY::RING) __nanosleep(64);
                 head = pos + agg;
+                s_head = head;
+                s_last_agg = agg;
+                s_alloc_it = it + 1;
                 if (it >= NQ) mbar_wait(&s_done[q], (it / NQ - 1) & 1);
                 s_pos = pos;
                 s_qt[q] = t;
@@ -679,6 +688,16 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
             for (uint32_t it = 0;; ++it) {
                 const int bi = it & 1;
                 if (it >= 2) mbar_wait(&s_free[bi], (it / 2 - 1) & 1);
+                // A claimed tile must never sit behind a full ring (which drains only
+                // as lookbacks complete), or lookbacks chain up across CTAs. Claim
+                // ahead only while the ring clearly has room for the tile being encoded
+                // and this one; otherwise wait until the previous tile holds its ring
+                // space (then nothing this tile waits on depends on a lookback).
+                while (it > 0) {
+                    const uint32_t last = s_last_agg, used = s_head - s_tail;
+                    if (used + 3 * last + 64 <= LY::RING || s_alloc_it >= it) break;
+                    __nanosleep(64);
+                }
                 const uint32_t tk = atomicAdd(ticket, 1u);
                 s_tkin[bi] = tk;
                 uint64_t *bar = &s_full[bi];

@@ -8,7 +8,9 @@ vp, u64, i32, dbl = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int, ctypes.c_dou
 lib.cszp2_compress.argtypes = [vp, u64, i32, dbl, i32, i32, vp, vp, vp]
 lib.cszp2_compress_bound.argtypes = [u64, i32]; lib.cszp2_compress_bound.restype = u64
 lib.cszp2_debug_set_trace.argtypes = [vp]
-for cfg in sys.argv[1:]:
+for arg in sys.argv[1:]:
+    cfg, _, mode = arg.partition(":")
+    enc = 0 if mode == "plain" else 1
     spec = CONFIGS[cfg]
     x = make_field(cfg, "cuda"); n = x.numel()
     T = -(-(-(-n // 32)) // 256)
@@ -18,7 +20,7 @@ for cfg in sys.argv[1:]:
     st = torch.cuda.current_stream().cuda_stream
     for rep in range(3):
         tr.zero_()
-        lib.cszp2_compress(ctypes.c_void_p(x.data_ptr()), n, 0, spec.ebs[-1], 1, 1, ctypes.c_void_p(out.data_ptr()), None, ctypes.c_void_p(st))
+        lib.cszp2_compress(ctypes.c_void_p(x.data_ptr()), n, 0, spec.ebs[-1], 1, enc, ctypes.c_void_p(out.data_ptr()), None, ctypes.c_void_p(st))
         torch.cuda.synchronize()
     a = tr.view(T, 8).cpu().numpy().astype(np.int64)
     t0 = a[:, 0][a[:, 0] > 0].min()
