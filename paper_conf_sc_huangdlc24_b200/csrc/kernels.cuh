@@ -169,6 +169,124 @@ __device__ __forceinline__ uint32_t ld_u32_unaligned(const uint8_t *base, uint32
     return __funnelshift_r(w[0], w[1], 8u * (pos & 3u));
 }
 
+// ------------------------------------------------------------------ bit-plane transposes
+// A 32x32 bit matrix in 32 registers (row r = A[r], column c = bit c) transposes
+// in five stages; stage s exchanges the s-bit off-diagonal blocks of every 2s x 2s
+// block (it swaps bit log2(s) of the row index with that of the column index, so the
+// stages commute). When only the first R = 2^M columns can be nonzero, the stages
+// s >= R reduce to merges A[i] |= A[i+s] << s (rows [s, 2s) become zero) and the
+// remaining ones touch rows [0, R) only. Cost per 32 values: R=1: 31 ops, 2: 35,
+// 4: 48, 8: 84, 16: 176, 32: 400 — against 64 per plane for a bit-serial pack.
+__host__ __device__ constexpr uint32_t stage_mask(int s) {
+    return s == 16 ? 0x0000FFFFu
+                   : (s == 8 ? 0x00FF00FFu : (s == 4 ? 0x0F0F0F0Fu : (s == 2 ? 0x33333333u : 0x55555555u)));
+}
+template <int S, int ROWS>
+__device__ __forceinline__ void swap_stage(uint32_t (&A)[32]) {
+#pragma unroll
+    for (int i = 0; i < ROWS; i++) {
+        if ((i & S) == 0) {
+            const uint32_t t = ((A[i] >> S) ^ A[i + S]) & stage_mask(S);
+            A[i + S] ^= t;
+            A[i] ^= t << S;
+        }
+    }
+}
+// values (bits < 2^M) -> planes: A[k] = sum_i bit_k(value_i) << i, k < 2^M
+template <int S>
+__device__ __forceinline__ void merge_stage(uint32_t (&A)[32]) {
+#pragma unroll
+    for (int i = 0; i < S; i++) A[i] |= A[i + S] << S;
+}
+template <int S>
+__device__ __forceinline__ void split_stage(uint32_t (&A)[32]) {
+#pragma unroll
+    for (int i = 0; i < S; i++) {
+        A[i + S] = (A[i] >> S) & stage_mask(S);
+        A[i] &= stage_mask(S);
+    }
+}
+template <int M>
+__device__ __forceinline__ void pack_planes(uint32_t (&A)[32]) {
+    constexpr int R = 1 << M;
+    if constexpr (R <= 16) merge_stage<16>(A);
+    if constexpr (R <= 8) merge_stage<8>(A);
+    if constexpr (R <= 4) merge_stage<4>(A);
+    if constexpr (R <= 2) merge_stage<2>(A);
+    if constexpr (R <= 1) merge_stage<1>(A);
+    if constexpr (M >= 5) swap_stage<16, R>(A);
+    if constexpr (M >= 4) swap_stage<8, R>(A);
+    if constexpr (M >= 3) swap_stage<4, R>(A);
+    if constexpr (M >= 2) swap_stage<2, R>(A);
+    if constexpr (M >= 1) swap_stage<1, R>(A);
+}
+// planes (rows >= fl zero, rows >= 2^M don't care) -> values: A[i] = sum_k bit_i(plane_k) << k
+template <int M>
+__device__ __forceinline__ void unpack_planes(uint32_t (&A)[32]) {
+    constexpr int R = 1 << M;
+    if constexpr (M >= 1) swap_stage<1, R>(A);
+    if constexpr (M >= 2) swap_stage<2, R>(A);
+    if constexpr (M >= 3) swap_stage<4, R>(A);
+    if constexpr (M >= 4) swap_stage<8, R>(A);
+    if constexpr (M >= 5) swap_stage<16, R>(A);
+    if constexpr (R <= 1) split_stage<1>(A);
+    if constexpr (R <= 2) split_stage<2>(A);
+    if constexpr (R <= 4) split_stage<4>(A);
+    if constexpr (R <= 8) split_stage<8>(A);
+    if constexpr (R <= 16) split_stage<16>(A);
+}
+// p ? a : b through selp, which the front end cannot turn into an indexed load
+__device__ __forceinline__ uint32_t opaque_select(bool p, uint32_t a, uint32_t b) {
+    uint32_t r;
+    asm("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %1, 0;\n\tselp.b32 %0, %2, %3, q;\n\t}"
+        : "=r"(r)
+        : "r"(static_cast<uint32_t>(p)), "r"(a), "r"(b));
+    return r;
+}
+// smallest M with fl <= 2^M (fl in 1..31)
+__device__ __forceinline__ int plane_log2(int fl) { return fl <= 1 ? 0 : 32 - __clz(fl - 1); }
+
+// One block's payload to smem at byte address `st` (any alignment): sign word, nob
+// outlier bytes, then planes A[0..fl). With P_-1 = the four header bytes just before
+// the plane region and r = its phase, every aligned word from (planes - r) on is
+// funnel(P_k-1, P_k, 8r) — wholly inside the block since the header is >= 4 bytes —
+// so the SIMT path is branch-free: <= 8 predicated header bytes, fl word stores and
+// <= 3 tail bytes (plain blocks, always 4-byte aligned, store whole words only).
+template <int R>
+__device__ __forceinline__ void stage_payload(uint8_t *base, uint32_t st, uint32_t sign,
+                                              uint32_t outl, int nob, int fl,
+                                              const uint32_t (&A)[32]) {
+    const uint64_t hdr = sign | (static_cast<uint64_t>(outl) << 32);
+    const uint32_t hb = 4u + nob;
+    const uint32_t ps = st + hb;  // plane region
+    const uint32_t r = fl ? (ps & 3u) : 0u;
+    const uint32_t nh = fl ? hb - r : hb;  // header bytes not covered by the word stream
+    if (nob == 0 && (st & 3u) == 0) {  // Plain: everything is whole aligned words
+        *reinterpret_cast<uint32_t *>(base + st) = sign;
+    } else {
+#pragma unroll
+        for (uint32_t j = 0; j < 8; j++)
+            if (j < nh) base[st + j] = static_cast<uint8_t>(hdr >> (8 * j));
+    }
+    if (fl == 0) return;
+    const uint32_t sh = 8u * r;
+    uint32_t *w = reinterpret_cast<uint32_t *>(base + ps - r);
+    uint32_t prev = static_cast<uint32_t>(hdr >> (8 * nob));  // P_-1
+    uint32_t top = A[0];
+#pragma unroll
+    for (int k = 0; k < R; k++) {
+        if (k < fl) {
+            w[k] = __funnelshift_l(prev, A[k], sh);
+            prev = A[k];
+        }
+        top = opaque_select(k < fl, A[k], top);
+    }
+    const uint32_t e = ps + 4u * fl;  // end of the payload
+#pragma unroll
+    for (uint32_t j = 0; j < 3; j++)
+        if (j < r) base[e - r + j] = static_cast<uint8_t>(top >> (32 - sh + 8 * j));
+}
+
 // ------------------------------------------------------------------ scans
 __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
 #pragma unroll
@@ -446,7 +564,7 @@ struct HdrStatic {
 // tile's aggregate appears within one load + encode of the claim.
 constexpr int NT_COMP = NT + 128;
 constexpr int LOADER_WARP = NT / 32;       // warp 8
-constexpr int RESOLVE_WARP = NT / 32 + 1;  // warps 9-10
+constexpr int RESOLVE_WARP = NT / 32 + 1;  // warp 9
 constexpr int NRESOLVE = 1;                // lookback warps (queue entries round-robin)
 constexpr int WRITER0 = NT + 64;           // first writer thread (warps 10-11)
 constexpr int NWRITER = NT_COMP - WRITER0; // 64 writer threads
@@ -654,25 +772,32 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
             if (active) out[g.O + b] = static_cast<uint8_t>(obyte);  // ❹ offset bytes
             named_sync(BAR_PROD, NT);  // s_pos visible
 
-            // ❷ payload staged in the ring at its tile-relative byte offset
-            if (size) {
-                uint8_t *p = ring + (s_pos % LY::RING) + my_excl;
-                st_u32_unaligned(p, sign);
-                p += 4;
-                if (OUTLIER && nob) {
-                    for (int j = 0; j < nob; j++) p[j] = static_cast<uint8_t>(a[0] >> (8 * j));
-                    p += nob;
-                    a[0] = 0;  // the outlier slot of every plane is 0
-                }
-                if (fl) {
-                    const int sh = 32 - fl;
-#pragma unroll
-                    for (int i = 0; i < L; i++) a[i] <<= sh;
-                    for (int kk = fl - 1; kk >= 0; kk--) {  // planes top-down, 2 ops per bit
-                        uint32_t w = 0;
-#pragma unroll
-                        for (int i = L - 1; i >= 0; i--) shift_bit_into(a[i], w);
-                        st_u32_unaligned(p + 4 * kk, w);
+            // ❷ payload staged in the ring at its tile-relative byte offset; bit planes
+            // by an in-register transpose sized to the warp's largest fixed length
+            {
+                const uint32_t st = (s_pos % LY::RING) + my_excl;
+                const uint32_t outl = a[0];
+                if (OUTLIER && nob) a[0] = 0;  // the outlier slot of every plane is 0
+                const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, static_cast<unsigned>(size ? fl : 0)));
+                if (size) {
+                    if (flw <= 1) {
+                        pack_planes<0>(a);
+                        stage_payload<1>(ring, st, sign, outl, nob, fl, a);
+                    } else if (flw <= 2) {
+                        pack_planes<1>(a);
+                        stage_payload<2>(ring, st, sign, outl, nob, fl, a);
+                    } else if (flw <= 4) {
+                        pack_planes<2>(a);
+                        stage_payload<4>(ring, st, sign, outl, nob, fl, a);
+                    } else if (flw <= 8) {
+                        pack_planes<3>(a);
+                        stage_payload<8>(ring, st, sign, outl, nob, fl, a);
+                    } else if (flw <= 16) {
+                        pack_planes<4>(a);
+                        stage_payload<16>(ring, st, sign, outl, nob, fl, a);
+                    } else {
+                        pack_planes<5>(a);
+                        stage_payload<32>(ring, st, sign, outl, nob, fl, a);
                     }
                 }
             }
@@ -765,13 +890,12 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
             write_payload(ring + (pos % LY::RING), out, dst0, agg, w, NWRITER);
             if (t == T_eff - 1) {  // last tile: pads, header, d_out_bytes
                 const uint64_t dst1 = dst0 + agg;
-                if (w >= 32 && w < 48) {  // zero pad after the payload
-                    const uint64_t o = dst1 + (w - 32);
+                __syncwarp();
+                if (w < 16) {  // zero pad after the payload
+                    const uint64_t o = dst1 + w;
                     if (o < roundup16(dst1)) out[o] = 0;
-                }
-                static_assert(NWRITER >= 64, "pads use writer threads 32..63");
-                if (w >= 48 && w < 64) {  // zero pad after the offset bytes
-                    const uint64_t o = g.O + g.nb + (w - 48);
+                } else if (w < 32) {  // zero pad after the offset bytes
+                    const uint64_t o = g.O + g.nb + (w - 16);
                     if (o < g.D) out[o] = 0;
                 }
                 if (w == 0) {
