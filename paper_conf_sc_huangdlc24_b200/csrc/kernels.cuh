@@ -287,6 +287,26 @@ __device__ __forceinline__ void stage_payload(uint8_t *base, uint32_t st, uint32
         if (j < r) base[e - r + j] = static_cast<uint8_t>(top >> (32 - sh + 8 * j));
 }
 
+// Planes 0..fl-1 of one block from smem at byte position `pos` (any alignment) into
+// A[0..R): rows >= fl are zeroed; each plane is a funnel of two aligned words.
+template <int R>
+__device__ __forceinline__ void load_planes(const uint8_t *base, uint32_t pos, uint32_t fl,
+                                            uint32_t (&A)[32]) {
+    const uint32_t *w = reinterpret_cast<const uint32_t *>(base + (pos & ~3u));
+    const uint32_t sh = 8u * (pos & 3u);
+    uint32_t lo = w[0];
+#pragma unroll
+    for (int k = 0; k < R; k++) {
+        uint32_t v = 0;
+        if (k < (int)fl) {
+            const uint32_t hi = w[k + 1];
+            v = __funnelshift_r(lo, hi, sh);
+            lo = hi;
+        }
+        A[k] = v;
+    }
+}
+
 // ------------------------------------------------------------------ scans
 __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
 #pragma unroll
@@ -1077,6 +1097,7 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) decompress_kernel(
 #pragma unroll
         for (int i = 0; i < L; i++) a[i] = 0;
         uint32_t sign = 0;
+        const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, size ? fl : 0u));
         if (size) {
             uint32_t pos = phase + my_excl;
             sign = ld_u32_unaligned(pbuf, pos);
@@ -1087,10 +1108,27 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) decompress_kernel(
                 if (nob < 4) outlier &= (1u << (8 * nob)) - 1u;
                 pos += nob;
             }
-            for (int k = static_cast<int>(fl) - 1; k >= 0; k--) {
-                uint32_t w = ld_u32_unaligned(pbuf, pos + 4 * k);
-#pragma unroll
-                for (int i = L - 1; i >= 0; i--) shift_bit_into(w, a[i]);
+            // planes -> values by an in-register transpose sized to the warp's max fl
+            if (flw > 0) {
+                if (flw <= 1) {
+                    load_planes<1>(pbuf, pos, fl, a);
+                    unpack_planes<0>(a);
+                } else if (flw <= 2) {
+                    load_planes<2>(pbuf, pos, fl, a);
+                    unpack_planes<1>(a);
+                } else if (flw <= 4) {
+                    load_planes<4>(pbuf, pos, fl, a);
+                    unpack_planes<2>(a);
+                } else if (flw <= 8) {
+                    load_planes<8>(pbuf, pos, fl, a);
+                    unpack_planes<3>(a);
+                } else if (flw <= 16) {
+                    load_planes<16>(pbuf, pos, fl, a);
+                    unpack_planes<4>(a);
+                } else {
+                    load_planes<32>(pbuf, pos, fl, a);
+                    unpack_planes<5>(a);
+                }
             }
             if (is_o) a[0] = outlier;
         }
