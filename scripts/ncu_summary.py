@@ -107,7 +107,7 @@ def main():
         rb, wb = d.get("dram__bytes_read.sum", 0), d.get("dram__bytes_write.sum", 0)
         md += [f"## {k}", "",
                f"- duration {t/1e3:.1f} us; DRAM read {rb/1e6:.1f} MB, write {wb/1e6:.1f} MB "
-               f"-> {(rb+wb)/t:.0f} GB/s; dram throughput {d.get('dram__throughput.avg.pct_of_peak_sustained_elapsed', 0):.1f}% of peak",
+               f"-> {(rb+wb)/t:.0f} GB/s",
                f"- issue active {d.get('smsp__issue_active.avg.pct_of_peak_sustained_active', 0):.1f}%, warps active "
                f"{d.get('sm__warps_active.avg.pct_of_peak_sustained_active', 0):.1f}%, "
                f"{d.get('launch__registers_per_thread', 0):.0f} regs/thread, grid {d.get('launch__grid_size', 0):.0f} x "
