@@ -247,32 +247,30 @@ __device__ __forceinline__ uint32_t opaque_select(bool p, uint32_t a, uint32_t b
 __device__ __forceinline__ int plane_log2(int fl) { return fl <= 1 ? 0 : 32 - __clz(fl - 1); }
 
 // One block's payload to smem at byte address `st` (any alignment): sign word, nob
-// outlier bytes, then planes A[0..fl). With P_-1 = the four header bytes just before
-// the plane region and r = its phase, every aligned word from (planes - r) on is
-// funnel(P_k-1, P_k, 8r) — wholly inside the block since the header is >= 4 bytes —
-// so the SIMT path is branch-free: <= 8 predicated header bytes, fl word stores and
-// <= 3 tail bytes (plain blocks, always 4-byte aligned, store whole words only).
+// outlier bytes, then planes A[0..fl). Let ps = st + 4 + nob (plane region), r = ps & 3
+// and P_k the 4 payload bytes at ps + 4k (P_-1, P_-2: header bytes before ps). Every
+// aligned word at ps - r + 4k is funnel(P_k-1, P_k, 8r); those wholly inside the block
+// (k = 0..fl-1, and k = -1 when nob >= r) are plain 32-bit stores, and only the <= 4
+// head and <= 3 tail bytes that share a word with a neighbouring block are written as
+// bytes. SIMT-uniform: no data-dependent branches.
 template <int R>
 __device__ __forceinline__ void stage_payload(uint8_t *base, uint32_t st, uint32_t sign,
                                               uint32_t outl, int nob, int fl,
                                               const uint32_t (&A)[32]) {
     const uint64_t hdr = sign | (static_cast<uint64_t>(outl) << 32);
-    const uint32_t hb = 4u + nob;
-    const uint32_t ps = st + hb;  // plane region
-    const uint32_t r = fl ? (ps & 3u) : 0u;
-    const uint32_t nh = fl ? hb - r : hb;  // header bytes not covered by the word stream
-    if (nob == 0 && (st & 3u) == 0) {  // Plain: everything is whole aligned words
-        *reinterpret_cast<uint32_t *>(base + st) = sign;
-    } else {
-#pragma unroll
-        for (uint32_t j = 0; j < 8; j++)
-            if (j < nh) base[st + j] = static_cast<uint8_t>(hdr >> (8 * j));
-    }
-    if (fl == 0) return;
+    const uint32_t ps = st + 4u + nob;
+    const uint32_t r = ps & 3u;
     const uint32_t sh = 8u * r;
-    uint32_t *w = reinterpret_cast<uint32_t *>(base + ps - r);
-    uint32_t prev = static_cast<uint32_t>(hdr >> (8 * nob));  // P_-1
-    uint32_t top = A[0];
+    const uint32_t pm1 = static_cast<uint32_t>(hdr >> (8 * nob));                // P_-1
+    const uint32_t pm2 = static_cast<uint32_t>(hdr << (32 - 8 * nob));           // P_-2 (top nob bytes)
+    uint32_t *w = reinterpret_cast<uint32_t *>(base + ps - r);                   // word k at w[k]
+    const bool wm1 = static_cast<uint32_t>(nob) >= r;
+    if (wm1) w[-1] = __funnelshift_l(pm2, pm1, sh);
+    const uint32_t head = (ps - r - (wm1 ? 4u : 0u)) - st;                         // 0..4 bytes
+#pragma unroll
+    for (uint32_t j = 0; j < 4; j++)
+        if (j < head) base[st + j] = static_cast<uint8_t>(hdr >> (8 * j));
+    uint32_t prev = pm1, top = pm1;
 #pragma unroll
     for (int k = 0; k < R; k++) {
         if (k < fl) {
@@ -832,7 +830,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
         if ((tid & 31) == 0) {
             for (uint32_t it = 0;; ++it) {
                 const int bi = it & 1;
-                if (it >= 2) mbar_wait(&s_free[bi], (it / 2 - 1) & 1);
+                if (it >= 2) mbar_wait_backoff(&s_free[bi], (it / 2 - 1) & 1, 100);
                 // A claimed tile must never sit behind a full ring (which drains only
                 // as lookbacks complete), or lookbacks chain up across CTAs. Claim
                 // ahead only while the ring clearly has room for the tile being encoded
@@ -875,7 +873,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
         const int lane = tid & 31;
         for (uint32_t it = warp - RESOLVE_WARP;; it += NRESOLVE) {
             const int q = it % NQ;
-            mbar_wait(&s_staged[q], (it / NQ) & 1);
+            mbar_wait_backoff(&s_staged[q], (it / NQ) & 1, 200);
             if (it >= s_end) {
                 if (lane == 0 && it == s_end) mbar_arrive(&s_resolved[q]);  // writer's end
                 break;
@@ -900,7 +898,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
             eb_from_header ? *reinterpret_cast<const volatile double *>(out + 32) : eb_abs_arg;
         for (uint32_t it = 0;; ++it) {
             const int q = it % NQ;
-            mbar_wait(&s_resolved[q], (it / NQ) & 1);
+            mbar_wait_backoff(&s_resolved[q], (it / NQ) & 1, 200);
             if (it >= s_end) break;
             const uint64_t t = s_qt[q];
             const uint64_t excl = s_qexcl[q];

@@ -69,6 +69,12 @@ __device__ __forceinline__ bool named_sync_or(uint32_t id, uint32_t n, bool v) {
     return r != 0;
 }
 
+// Wait with a nanosleep back-off between polls: for warps whose wake-up latency
+// matters less than the issue slots their polling would take from busy warps.
+__device__ __forceinline__ void mbar_wait_backoff(uint64_t *bar, uint32_t parity, uint32_t ns) {
+    while (!mbar_try_wait(bar, parity)) __nanosleep(ns);
+}
+
 // ---------------------------------------------------------------- TMA
 // 2D tensor tile global -> shared (completes on an mbarrier).
 __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, int x, int y,
