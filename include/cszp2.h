@@ -90,6 +90,14 @@ int cszp2_compress_prepare(const void *d_in, uint64_t n, int dtype, double eb, i
 int cszp2_compress_encode(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
                           int enc_mode, void *d_out, uint64_t *d_out_bytes, void *stream);
 
+/* cszp2_compress_encode with ablation flags (same stream bytes either way):
+ *  CSZP2_FLAG_CHAINED_SCAN: replace the decoupled lookback by the plain chained
+ *  scan it improves on (Fig 12 left; the Fig 17 comparison). */
+#define CSZP2_FLAG_CHAINED_SCAN 1u
+int cszp2_compress_encode_ex(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
+                             int enc_mode, void *d_out, uint64_t *d_out_bytes, unsigned flags,
+                             void *stream);
+
 /* Decompression (❸ locate → ❹ → ❷ → ❶ in one kernel).
  *  d_cmp    : a stream produced by cszp2_compress for the same (n, dtype),
  *             device, 16-byte aligned.
@@ -100,6 +108,15 @@ int cszp2_compress_encode(const void *d_in, uint64_t n, int dtype, double eb, in
  *             caller zeroes it beforehand. */
 int cszp2_decompress(const void *d_cmp, void *d_out, uint64_t n, int dtype, int *d_status,
                      void *stream);
+
+/* Random-access decompression (§VI-B): decode only the values
+ * [first, first + count) of a stream of n values into d_out[0 .. count)
+ * (device, any 4/8-byte alignment). Only the tiles (256 blocks = 8192 values)
+ * covering the range are read; each is located in O(1) through the stream's
+ * tile index (FORMAT.md §2). d_status as in cszp2_decompress. Errors: ARG if
+ * the range exceeds n. */
+int cszp2_decompress_range(const void *d_cmp, uint64_t n, int dtype, uint64_t first,
+                           uint64_t count, void *d_out, int *d_status, void *stream);
 
 /* Copy the 64-byte header of a device stream to the host and decode it.
  * Synchronises `stream`. */

@@ -60,8 +60,10 @@ def _load():
     L.cszp2_compress.argtypes = sig
     L.cszp2_compress_encode.argtypes = sig
     L.cszp2_compress_prepare.argtypes = [vp, u64, i32, dbl, i32, vp, vp]
+    L.cszp2_compress_encode_ex.argtypes = [vp, u64, i32, dbl, i32, i32, vp, vp, ctypes.c_uint, vp]
     L.cszp2_decompress.argtypes = [vp, vp, u64, i32, vp, vp]
     L.cszp2_read_header.argtypes = [vp, ctypes.POINTER(Header), vp]
+    L.cszp2_decompress_range.argtypes = [vp, u64, i32, u64, u64, vp, vp, vp]
     L.cszp2_compress_host.argtypes = [vp, u64, i32, dbl, i32, i32, vp, vp, vp, u64,
                                       ctypes.POINTER(ctypes.c_uint64), vp]
     L.cszp2_decompress_host.argtypes = [vp, u64, vp, vp, vp, u64, i32, vp, vp]
@@ -74,7 +76,8 @@ _lib = _load()
 LIBRARY_PATH = _LIB_PATH
 EXPORTED = (
     "cszp2_compress_bound", "cszp2_compress", "cszp2_compress_prepare", "cszp2_compress_encode",
-    "cszp2_decompress", "cszp2_read_header", "cszp2_compress_host", "cszp2_decompress_host",
+    "cszp2_compress_encode_ex",
+    "cszp2_decompress", "cszp2_decompress_range", "cszp2_read_header", "cszp2_compress_host", "cszp2_decompress_host",
     "cszp2_container_index", "cszp2_version",
 )
 
@@ -140,6 +143,16 @@ def compress_encode(x, eb, eb_mode, enc_mode, out, out_bytes=None, stream=None):
     _check("cszp2_compress_encode", rc)
 
 
+FLAG_CHAINED_SCAN = 1
+
+
+def compress_encode_ex(x, eb, eb_mode, enc_mode, out, out_bytes=None, flags=0, stream=None):
+    """compress_encode with ablation flags (FLAG_CHAINED_SCAN: plain chained scan)."""
+    rc = _lib.cszp2_compress_encode_ex(_ptr(x), x.numel(), _DT[x.dtype], float(eb), _EB[eb_mode],
+                                       _ENC[enc_mode], _ptr(out), _ptr(out_bytes), flags, _stream(stream))
+    _check("cszp2_compress_encode_ex", rc)
+
+
 def decompress(cmp: torch.Tensor, n: int, dtype=torch.float32, out=None, status=None, stream=None):
     """Decompress a device stream into n values. `status` (optional device
     int32 tensor, zeroed by the caller) receives CSZP2_ERR_FORMAT/RANGE bits."""
@@ -148,6 +161,18 @@ def decompress(cmp: torch.Tensor, n: int, dtype=torch.float32, out=None, status=
         out = torch.empty(n, dtype=dtype, device=cmp.device)
     rc = _lib.cszp2_decompress(_ptr(cmp), _ptr(out), n, _DT[out.dtype], _ptr(status), _stream(stream))
     _check("cszp2_decompress", rc)
+    return out
+
+
+def decompress_range(cmp: torch.Tensor, n: int, first: int, count: int, dtype=torch.float32, out=None,
+                     status=None, stream=None):
+    """Random access: values [first, first+count) of an n-value stream."""
+    _need_cuda(cmp, out, status)
+    if out is None:
+        out = torch.empty(count, dtype=dtype, device=cmp.device)
+    rc = _lib.cszp2_decompress_range(_ptr(cmp), n, _DT[out.dtype], first, count, _ptr(out), _ptr(status),
+                                     _stream(stream))
+    _check("cszp2_decompress_range", rc)
     return out
 
 

@@ -127,7 +127,7 @@ int launch_minmax(const void *d_in, uint64_t n, double lambda, void *d_out, cuda
 
 template <typename T, bool OUTLIER>
 int launch_compress(const void *d_in, const Geom &g, double eb, int eb_mode, int enc_mode,
-                    void *d_out, uint64_t *d_out_bytes, cudaStream_t st) {
+                    void *d_out, uint64_t *d_out_bytes, cudaStream_t st, unsigned flags) {
     static std::once_flag once;
     static int attr_rc = CSZP2_OK;
     static int grid_cache = 0;
@@ -144,6 +144,7 @@ int launch_compress(const void *d_in, const Geom &g, double eb, int eb_mode, int
                (static_cast<uint32_t>(enc_mode) << 16) | (5u << 24);
     hs.eb_mode = static_cast<uint32_t>(eb_mode);
     hs.eb_user = eb;
+    hs.flags = flags;
     compress_kernel<T, OUTLIER><<<grid, NT_COMP, smem, st>>>(
         map, static_cast<const T *>(d_in), g, eb, eb_mode == CSZP2_EB_REL ? 1 : 0,
         static_cast<uint8_t *>(d_out), ticket, d_out_bytes, hs);
@@ -200,19 +201,28 @@ int cszp2_compress_prepare(const void *d_in, uint64_t n, int dtype, double eb, i
     return CSZP2_OK;
 }
 
-int cszp2_compress_encode(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
-                          int enc_mode, void *d_out, uint64_t *d_out_bytes, void *stream) {
+int cszp2_compress_encode_ex(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
+                             int enc_mode, void *d_out, uint64_t *d_out_bytes, unsigned flags,
+                             void *stream) {
     int rc = check_compress_args(d_in, n, dtype, eb, eb_mode, d_out);
     if (rc) return rc;
     if (enc_mode != CSZP2_ENC_PLAIN && enc_mode != CSZP2_ENC_OUTLIER) return CSZP2_ERR_ARG;
+    if (flags & ~1u) return CSZP2_ERR_ARG;
     Geom g = geometry(n);
+    cudaStream_t st = S(stream);
     if (dtype == CSZP2_F32)
         return enc_mode == CSZP2_ENC_OUTLIER
-                   ? launch_compress<float, true>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, S(stream))
-                   : launch_compress<float, false>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, S(stream));
+                   ? launch_compress<float, true>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags)
+                   : launch_compress<float, false>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags);
     return enc_mode == CSZP2_ENC_OUTLIER
-               ? launch_compress<double, true>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, S(stream))
-               : launch_compress<double, false>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, S(stream));
+               ? launch_compress<double, true>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags)
+               : launch_compress<double, false>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags);
+}
+
+int cszp2_compress_encode(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
+                          int enc_mode, void *d_out, uint64_t *d_out_bytes, void *stream) {
+    return cszp2_compress_encode_ex(d_in, n, dtype, eb, eb_mode, enc_mode, d_out, d_out_bytes, 0u,
+                                    stream);
 }
 
 int cszp2_compress(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode, int enc_mode,
@@ -231,6 +241,23 @@ int cszp2_decompress(const void *d_cmp, void *d_out, uint64_t n, int dtype, int 
     Geom g = geometry(n);
     return dtype == CSZP2_F32 ? launch_decompress<float>(d_cmp, d_out, g, d_status, S(stream))
                               : launch_decompress<double>(d_cmp, d_out, g, d_status, S(stream));
+}
+
+int cszp2_decompress_range(const void *d_cmp, uint64_t n, int dtype, uint64_t first,
+                           uint64_t count, void *d_out, int *d_status, void *stream) {
+    if (!wsize(dtype) || !d_cmp || (!d_out && count)) return CSZP2_ERR_ARG;
+    if (!aligned16(d_cmp) || n > (1ull << 40) || first > n || count > n - first) return CSZP2_ERR_ARG;
+    if (count == 0) return CSZP2_OK;
+    Geom g = geometry(n);
+    const uint64_t t0 = (first / L) / BPT, t1 = ((first + count - 1) / L) / BPT;
+    const unsigned grid = static_cast<unsigned>(t1 - t0 + 1);
+    if (dtype == CSZP2_F32)
+        decompress_range_kernel<float><<<grid, NT, 0, S(stream)>>>(
+            static_cast<const uint8_t *>(d_cmp), static_cast<float *>(d_out), g, first, count, t0, d_status);
+    else
+        decompress_range_kernel<double><<<grid, NT, 0, S(stream)>>>(
+            static_cast<const uint8_t *>(d_cmp), static_cast<double *>(d_out), g, first, count, t0, d_status);
+    return launch_status();
 }
 
 int cszp2_read_header(const void *d_cmp, cszp2_header *h, void *stream) {

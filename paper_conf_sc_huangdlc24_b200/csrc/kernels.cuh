@@ -443,6 +443,28 @@ __device__ __forceinline__ uint64_t lookback(uint64_t *index, uint64_t t, uint64
     return lookback_finish(index, t, agg, bad, w, range_out);
 }
 
+// Ablation (NEXT #2): the plain chained scan that decoupled lookback replaces
+// (Fig 12 left) — wait until the immediate predecessor holds its
+// inclusive prefix, then publish this tile's.
+__device__ __forceinline__ uint64_t chained_prefix(uint64_t *index, uint64_t t, uint64_t agg,
+                                                   bool bad, bool *range_out) {
+    const int lane = threadIdx.x & 31;
+    uint64_t d = 0;
+    if (lane == 0) {
+        d = ld_relaxed_u64(&index[t - 1]);
+        while ((d >> 62) != 2) {
+            __nanosleep(32);
+            d = ld_relaxed_u64(&index[t - 1]);
+        }
+    }
+    d = __shfl_sync(0xffffffffu, d, 0);
+    const uint64_t rbits = (d & BIT_RANGE) | (bad ? BIT_RANGE : 0);
+    const uint64_t excl = d & VAL61;
+    if (lane == 0) st_relaxed_u64(&index[t], FLAG_P | rbits | (excl + agg));
+    *range_out = rbits != 0;
+    return excl;
+}
+
 // ------------------------------------------------------------------ REL: min/max
 __device__ __forceinline__ uint32_t sortable(float x) {
     uint32_t u = __float_as_uint(x);
@@ -562,6 +584,7 @@ struct HdrStatic {
     uint32_t word1;    // header bytes 4..7: version, dtype, enc_mode, log2L
     uint32_t eb_mode;  // header byte 8
     double eb_user;    // header bytes 24..31
+    uint32_t flags;    // CSZP2_FLAG_* (ablations)
 };
 
 // Warp-specialised compression CTA (NT_COMP = 384 threads = 12 warps):
@@ -883,7 +906,13 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
             const bool bad = s_qbad[q];
             if (lane == 0) TRACE(t, 6, gtimer());
             bool rng = bad;
-            const uint64_t e = (g.T && t > 0) ? lookback(index, t, agg, bad, &rng) : 0;
+            uint64_t e = 0;
+            if (g.T && t > 0) {
+                if (hs.flags & 1u)  // ablation: plain chained scan (Fig 12 left)
+                    e = chained_prefix(index, t, agg, bad, &rng);
+                else
+                    e = lookback(index, t, agg, bad, &rng);
+            }
             if (lane == 0) {
                 s_qexcl[q] = e;
                 s_qrng[q] = rng;
@@ -939,6 +968,83 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
             }
         }
     }
+}
+
+// ------------------------------------------------------------------ block decode
+// ❷⁻¹ + inverse Lorenzo + ❶⁻¹ of one block whose payload starts at byte `pos` of the
+// shared buffer `pbuf`: sign field, outlier, bit planes (in-register
+// transpose sized to the warp's largest fixed length), q_i = q_{i-1} + d_i,
+// x_i = (T)q_i * s. Warp-collective: every lane of the warp must call it.
+template <typename T>
+__device__ __forceinline__ void decode_block(const uint8_t *pbuf, uint32_t pos, uint32_t obyte,
+                                             uint32_t size, T s, T (&x)[L]) {
+    const uint32_t fl = obyte & 31u;
+    const bool is_o = (obyte & 0x80u) != 0;
+    const uint32_t nob = is_o ? ((obyte >> 5) & 3u) + 1u : 0u;
+    uint32_t a[L];
+#pragma unroll
+    for (int i = 0; i < L; i++) a[i] = 0;
+    uint32_t sign = 0;
+    const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, size ? fl : 0u));
+    if (size) {
+        sign = ld_u32_unaligned(pbuf, pos);
+        pos += 4;
+        uint32_t outlier = 0;
+        if (is_o) {
+            outlier = ld_u32_unaligned(pbuf, pos);
+            if (nob < 4) outlier &= (1u << (8 * nob)) - 1u;
+            pos += nob;
+        }
+        if (flw > 0) {
+            if (flw <= 1) {
+                load_planes<1>(pbuf, pos, fl, a);
+                unpack_planes<0>(a);
+            } else if (flw <= 2) {
+                load_planes<2>(pbuf, pos, fl, a);
+                unpack_planes<1>(a);
+            } else if (flw <= 4) {
+                load_planes<4>(pbuf, pos, fl, a);
+                unpack_planes<2>(a);
+            } else if (flw <= 8) {
+                load_planes<8>(pbuf, pos, fl, a);
+                unpack_planes<3>(a);
+            } else if (flw <= 16) {
+                load_planes<16>(pbuf, pos, fl, a);
+                unpack_planes<4>(a);
+            } else {
+                load_planes<32>(pbuf, pos, fl, a);
+                unpack_planes<5>(a);
+            }
+        }
+        if (is_o) a[0] = outlier;
+    }
+    int qv = 0;
+#pragma unroll
+    for (int i = 0; i < L; i++) {
+        const int d = ((sign >> i) & 1u) ? -static_cast<int>(a[i]) : static_cast<int>(a[i]);
+        qv += d;
+        x[i] = dequantize(qv, s);
+    }
+}
+
+// Header checks shared by the decompression kernels (FORMAT.md §3): returns 0, or
+// ST_FORMAT / ST_RANGE; *eb and *pb receive eb_abs and the payload byte count.
+template <typename T>
+__device__ __forceinline__ int check_header(const uint8_t *cmp, const Geom &g, double *eb,
+                                            uint64_t *pb) {
+    const uint64_t *h = reinterpret_cast<const uint64_t *>(cmp);
+    const uint64_t h0 = h[0], h1 = h[1];
+    int err = 0;
+    const uint32_t want1 = 1u | (static_cast<uint32_t>(Traits<T>::DTYPE) << 8) | (5u << 24);
+    if ((h0 & 0xFFFFFFFFu) != MAGIC || ((h0 >> 32) & 0xFF00FFFFu) != want1 ||
+        ((h1 >> 16) & 0xFFFFu) != BPT || h[2] != g.n)
+        err = ST_FORMAT;
+    else if (((h1 >> 8) & 0xFF) != 0)
+        err = ((h1 >> 8) & 0xFF) == ST_RANGE ? ST_RANGE : ST_FORMAT;
+    *pb = h[5];
+    if (!err && h[6] != roundup16(g.D + *pb)) err = ST_FORMAT;
+    *eb = __longlong_as_double(static_cast<long long>(h[4]));
+    return err;
 }
 
 // ------------------------------------------------------------------ decompression
@@ -1002,18 +1108,9 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) decompress_kernel(
     uint64_t t = blockIdx.x;
     if (tid == 0) {
         // header checks (FORMAT.md §3) — once per CTA
-        const uint64_t *h = reinterpret_cast<const uint64_t *>(cmp);
-        const uint64_t h0 = h[0], h1 = h[1];
-        int err = 0;
-        const uint32_t want1 = 1u | (static_cast<uint32_t>(Traits<T>::DTYPE) << 8) | (5u << 24);
-        if ((h0 & 0xFFFFFFFFu) != MAGIC || ((h0 >> 32) & 0xFF00FFFFu) != want1 ||
-            ((h1 >> 16) & 0xFFFFu) != BPT || h[2] != g.n)
-            err = ST_FORMAT;
-        else if (((h1 >> 8) & 0xFF) != 0)
-            err = ((h1 >> 8) & 0xFF) == ST_RANGE ? ST_RANGE : ST_FORMAT;
-        pb_hdr = h[5];
-        if (!err && h[6] != roundup16(g.D + pb_hdr)) err = ST_FORMAT;
-        s_eb = __longlong_as_double(static_cast<long long>(h[4]));
+        double eb;
+        int err = check_header<T>(cmp, g, &eb, &pb_hdr);
+        s_eb = eb;
         s_err = err;
         mbar_init(&s_bar[0], 1);
         mbar_init(&s_bar[1], 1);
@@ -1088,57 +1185,10 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) decompress_kernel(
         }
         mbar_wait(&s_bar[cur], (it >> 1) & 1);
 
-        // ---- ❷⁻¹ decode: sign field, outlier, bit planes (top plane first)
-        const uint8_t *pbuf = pbufs + cur * PBUF_BYTES;
-        const uint32_t phase = static_cast<uint32_t>((g.D + s_excl[cur]) & 15u);
-        uint32_t a[L];
-#pragma unroll
-        for (int i = 0; i < L; i++) a[i] = 0;
-        uint32_t sign = 0;
-        const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, size ? fl : 0u));
-        if (size) {
-            uint32_t pos = phase + my_excl;
-            sign = ld_u32_unaligned(pbuf, pos);
-            pos += 4;
-            uint32_t outlier = 0;
-            if (is_o) {
-                outlier = ld_u32_unaligned(pbuf, pos);
-                if (nob < 4) outlier &= (1u << (8 * nob)) - 1u;
-                pos += nob;
-            }
-            // planes -> values by an in-register transpose sized to the warp's max fl
-            if (flw > 0) {
-                if (flw <= 1) {
-                    load_planes<1>(pbuf, pos, fl, a);
-                    unpack_planes<0>(a);
-                } else if (flw <= 2) {
-                    load_planes<2>(pbuf, pos, fl, a);
-                    unpack_planes<1>(a);
-                } else if (flw <= 4) {
-                    load_planes<4>(pbuf, pos, fl, a);
-                    unpack_planes<2>(a);
-                } else if (flw <= 8) {
-                    load_planes<8>(pbuf, pos, fl, a);
-                    unpack_planes<3>(a);
-                } else if (flw <= 16) {
-                    load_planes<16>(pbuf, pos, fl, a);
-                    unpack_planes<4>(a);
-                } else {
-                    load_planes<32>(pbuf, pos, fl, a);
-                    unpack_planes<5>(a);
-                }
-            }
-            if (is_o) a[0] = outlier;
-        }
-        // ---- inverse Lorenzo (prefix sum) + ❶⁻¹ dequantization
+        // ---- ❷⁻¹ decode, inverse Lorenzo, ❶⁻¹ dequantization
         T x[L];
-        int qv = 0;
-#pragma unroll
-        for (int i = 0; i < L; i++) {
-            const int d = ((sign >> i) & 1u) ? -static_cast<int>(a[i]) : static_cast<int>(a[i]);
-            qv += d;
-            x[i] = dequantize(qv, K.s);
-        }
+        decode_block(pbufs + cur * PBUF_BYTES,
+                     static_cast<uint32_t>((g.D + s_excl[cur]) & 15u) + my_excl, obyte, size, K.s, x);
         if (tid == 0) bulk_wait_read0();  // the previous tile's store has read ostage
         __syncthreads();
         const bool full = b < g.nfull;
@@ -1168,6 +1218,89 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) decompress_kernel(
     if (tid == 0) {
         bulk_wait_read0();
         if (err && d_status) atomicOr(d_status, err);
+    }
+}
+
+// ------------------------------------------------------------------ random access
+// Random-access decompression (§VI-B): values [first, first + count) of the
+// stream, written to out[0 .. count). One CTA per tile covering the range; each tile is
+// located in O(1) from the persisted index (R-14), so no scan over earlier tiles runs.
+template <typename T>
+__global__ void __launch_bounds__(NT) decompress_range_kernel(const uint8_t *__restrict__ cmp,
+                                                              T *__restrict__ out, const Geom g,
+                                                              uint64_t first, uint64_t count,
+                                                              uint64_t t_begin,
+                                                              int *__restrict__ d_status) {
+    __shared__ __align__(16) uint8_t pbuf[PBUF_BYTES];
+    __shared__ uint64_t s_bar;
+    __shared__ uint32_t s_warp[NT / 32];
+    __shared__ uint64_t s_excl;
+    __shared__ uint32_t s_bytes;
+    __shared__ double s_eb;
+    __shared__ int s_err;
+    const int tid = threadIdx.x;
+    const uint64_t t = t_begin + blockIdx.x;
+    if (tid == 0) {
+        double eb;
+        uint64_t pb;
+        int err = check_header<T>(cmp, g, &eb, &pb);
+        uint64_t e = 0, i = 0;
+        if (!err) {
+            const uint64_t *index = reinterpret_cast<const uint64_t *>(cmp) + 8;
+            const uint64_t dp = t ? index[t - 1] : FLAG_P, di = index[t];
+            e = dp & VAL_MASK;
+            i = di & VAL_MASK;
+            if ((dp >> 61) != 4 || (di >> 61) != 4 || i < e || i > pb ||
+                i - e > static_cast<uint64_t>(BPT) * 4 * L)
+                err = ST_FORMAT;
+        }
+        s_err = err;
+        s_eb = eb;
+        s_excl = e;
+        s_bytes = static_cast<uint32_t>(i - e);
+        mbar_init(&s_bar, 1);
+        fence_mbar_init();
+        if (!err) {
+            if (i > e) {
+                const uint64_t src0 = (g.D + e) & ~uint64_t(15);
+                const uint32_t len = static_cast<uint32_t>(roundup16(g.D + i) - src0);
+                mbar_expect_tx(&s_bar, len);
+                bulk_load(pbuf, cmp + src0, len, &s_bar);
+            } else {
+                mbar_expect_tx(&s_bar, 0);
+            }
+        }
+    }
+    __syncthreads();
+    if (s_err) {
+        if (tid == 0 && d_status) atomicOr(d_status, s_err);
+        return;
+    }
+    const uint64_t b = t * BPT + tid;
+    const bool active = b < g.nb;
+    const uint32_t obyte = active ? cmp[g.O + b] : 0u;
+    const uint32_t fl = obyte & 31u;
+    const bool is_o = (obyte & 0x80u) != 0;
+    const uint32_t nob = is_o ? ((obyte >> 5) & 3u) + 1u : 0u;
+    bool bad = (!is_o && (obyte & 0x60u));
+    const uint32_t size = is_o ? 4u + nob + 4u * fl : (fl ? 4u * (1u + fl) : 0u);
+    uint32_t agg;
+    const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg);
+    bad |= (tid == 0 && agg != s_bytes);
+    const bool any_bad = __syncthreads_or(bad);
+    mbar_wait(&s_bar, 0);
+    if (any_bad) {
+        if (tid == 0 && d_status) atomicOr(d_status, ST_FORMAT);
+        return;
+    }
+    const auto K = make_consts(s_eb, static_cast<T *>(nullptr));
+    T x[L];
+    decode_block(pbuf, static_cast<uint32_t>((g.D + s_excl) & 15u) + my_excl, obyte, size, K.s, x);
+    const uint64_t v0 = b * L, last = first + count;
+#pragma unroll
+    for (int i = 0; i < L; i++) {
+        const uint64_t v = v0 + i;
+        if (v >= first && v < last && v < g.n) out[v - first] = x[i];
     }
 }
 

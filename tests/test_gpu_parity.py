@@ -153,6 +153,46 @@ def test_decompress_rejects_corrupt_streams():
     assert status(bad) == 4
 
 
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_random_access_ranges(dtype):
+    """NEXT #1, random access: any value range decodes to exactly the
+    oracle's values, touching only the tiles that cover it."""
+    rng = np.random.default_rng(21)
+    n = 8192 * 5 + 32 * 3 + 13
+    xh = (np.cumsum(rng.standard_normal(n)) * 0.7).astype(dtype)
+    x = torch.from_numpy(xh).to(DEV)
+    out, total = gpu_compress(x, 1e-3, "rel", "outlier")
+    ref, _ = oracle.compress(xh, 1e-3, oracle.REL, oracle.OUTLIER)
+    yr, _ = oracle.decompress(ref, n, dtype)
+    iv = np.uint32 if dtype == np.float32 else np.uint64
+    cases = [(0, 1), (0, 32), (5, 27), (31, 2), (8191, 2), (8190, 8200), (n - 13, 13), (n - 1, 1), (0, n),
+             (12345, 1000)] + [(int(a), int(rng.integers(1, 5000))) for a in rng.integers(0, n - 5000, 6)]
+    for first, count in cases:
+        st = torch.zeros(1, dtype=torch.int32, device=DEV)
+        y = cz.decompress_range(out, n, first, count, x.dtype, status=st)
+        torch.cuda.synchronize()
+        assert int(st.item()) == 0
+        np.testing.assert_array_equal(y.cpu().numpy().view(iv), yr[first:first + count].view(iv))
+    with pytest.raises(cz.CszpError):
+        cz.decompress_range(out, n, n - 1, 2, x.dtype)
+
+
+@pytest.mark.parametrize("enc", ["plain", "outlier"])
+def test_chained_scan_ablation_same_stream(enc):
+    """NEXT #2: the chained-scan ablation must emit the identical stream."""
+    rng = np.random.default_rng(4)
+    xh = np.cumsum(rng.standard_normal(8192 * 40 + 77)).astype(np.float32)
+    x = torch.from_numpy(xh).to(DEV)
+    a, ta = gpu_compress(x, 1e-3, "rel", enc)
+    b = torch.full_like(a, 0x55)
+    nb = torch.zeros(1, dtype=torch.int64, device=DEV)
+    cz.compress_prepare(x, 1e-3, "rel", b)
+    cz.compress_encode_ex(x, 1e-3, "rel", enc, b, nb, flags=cz.FLAG_CHAINED_SCAN)
+    torch.cuda.synchronize()
+    assert int(nb.item()) == ta
+    assert torch.equal(a[:ta], b[:ta])
+
+
 def test_container_index():
     sizes = torch.tensor([100, 0, 37, 5], dtype=torch.int64, device=DEV)
     off = cz.container_index(sizes)
