@@ -1052,26 +1052,31 @@ constexpr uint32_t PBUF_BYTES = BPT * 4 * L + 128;  // max tile payload + alignm
 
 template <typename T>
 constexpr int decompress_smem_bytes() {
-    return Traits<T>::TILE_BYTES + 2 * PBUF_BYTES + 1024;
+    return Traits<T>::TILE_BYTES + PBUF_BYTES + 1024;
 }
 
 // Persistent decompression kernel: CTA c decodes tiles c, c+G, c+2G, ... The
 // persisted tile index locates every tile in O(1) (no inter-CTA waiting), so the
 // next tile's index words, offset bytes and payload (1D bulk TMA) are fetched
 // while the current tile is decoded and stored (2D tensor TMA, 128B swizzle).
+// Payloads land in one 32 KiB ring, the next tile's right behind the current one
+// (at useful compression ratios both fit, so the fetch overlaps the decode); only
+// when they do not is the fetch deferred until the current tile is decoded. One
+// payload buffer instead of two fits three CTAs per SM for f32.
 template <typename T>
-__global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) decompress_kernel(const __grid_constant__ CUtensorMap tmap,
+__global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 3 : 2) decompress_kernel(const __grid_constant__ CUtensorMap tmap,
                                                            const uint8_t *__restrict__ cmp,
                                                            T *__restrict__ out, const Geom g,
                                                            int *__restrict__ d_status) {
     extern __shared__ uint8_t smem_raw[];
     uint8_t *ostage = reinterpret_cast<uint8_t *>(
         (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    uint8_t *pbufs = ostage + Traits<T>::TILE_BYTES;
+    uint8_t *ring = ostage + Traits<T>::TILE_BYTES;
     __shared__ uint64_t s_bar[2];
     __shared__ uint32_t s_warp[NT / 32];
     __shared__ uint64_t s_excl[2];
     __shared__ uint32_t s_bytes[2];
+    __shared__ uint32_t s_rpos[2];  // ring position of each slot's payload
     __shared__ double s_eb;
     __shared__ int s_err;
 
@@ -1085,8 +1090,14 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) decompress_kernel(
     uint64_t pb_hdr = 0;   // payload bytes from the header
     bool pending = false;  // a payload prefetch is in flight
 
-    // thread 0: tile meta from two index words -> smem slot, start its payload TMA
-    auto launch = [&](uint64_t tt, uint64_t dp, uint64_t di, int bi) {
+    // thread 0 ring state: [r_pos, r_pos + r_len) holds the current slot's payload
+    uint32_t r_pos = 0, r_len = 0;
+    bool deferred = false;  // next slot's payload waits for the ring to empty
+
+    // thread 0: tile meta from two index words -> smem slot; start its payload TMA
+    // into the ring (behind the current payload, else at 0 if that end is free) or
+    // defer it (returns false) when neither fits yet.
+    auto launch = [&](uint64_t dp, uint64_t di, int bi, bool ring_empty) -> bool {
         const uint64_t e = dp & VAL_MASK, i = di & VAL_MASK;  // bit 61 is 0 in a valid stream
         uint32_t bytes = BAD_BYTES;
         if ((dp >> 61) == 4 && (di >> 61) == 4 && i >= e && i <= pb_hdr &&
@@ -1097,12 +1108,26 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) decompress_kernel(
         if (bytes != BAD_BYTES && bytes) {
             const uint64_t src0 = (g.D + e) & ~uint64_t(15);
             const uint32_t len = static_cast<uint32_t>(roundup16(g.D + e + bytes) - src0);
+            uint32_t pos;
+            if (ring_empty)
+                pos = 0;
+            else if (r_pos + r_len + len <= PBUF_BYTES - 16)
+                pos = r_pos + r_len;
+            else if (len + 16 <= r_pos)
+                pos = 0;
+            else
+                return false;
+            s_rpos[bi] = pos;
+            r_pos = pos;
+            r_len = len;
             mbar_expect_tx(&s_bar[bi], len);
-            bulk_load(pbufs + bi * PBUF_BYTES, cmp + src0, len, &s_bar[bi]);
+            bulk_load(ring + pos, cmp + src0, len, &s_bar[bi]);
         } else {
+            s_rpos[bi] = 0;
+            r_len = 0;
             mbar_expect_tx(&s_bar[bi], 0);
         }
-        (void)tt;
+        return true;
     };
 
     uint64_t t = blockIdx.x;
@@ -1116,7 +1141,7 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) decompress_kernel(
         mbar_init(&s_bar[1], 1);
         fence_mbar_init();
         if (!err && t < g.T) {
-            launch(t, t ? index[t - 1] : FLAG_P, index[t], 0);
+            launch(t ? index[t - 1] : FLAG_P, index[t], 0, true);
             pending = true;
             const uint64_t t2 = t + G;
             if (t2 < g.T) {
@@ -1143,11 +1168,15 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) decompress_kernel(
     for (uint32_t it = 0; t < g.T; ++it, t += G) {
         const int cur = it & 1;
         const uint64_t tn = t + G;
+        uint64_t nraw_p = 0, nraw_i = 0;  // thread 0: the next tile's words if deferred
         if (tid == 0) {
             pending = false;
+            deferred = false;
             if (tn < g.T) {  // payload of the next tile streams in during this one
-                launch(tn, raw_p, raw_i, cur ^ 1);
-                pending = true;
+                nraw_p = raw_p;
+                nraw_i = raw_i;
+                deferred = !launch(raw_p, raw_i, cur ^ 1, false);
+                pending = !deferred;
                 const uint64_t t2 = tn + G;
                 if (t2 < g.T) {
                     raw_p = index[t2 - 1];
@@ -1187,10 +1216,14 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 2 : 1) decompress_kernel(
 
         // ---- ❷⁻¹ decode, inverse Lorenzo, ❶⁻¹ dequantization
         T x[L];
-        decode_block(pbufs + cur * PBUF_BYTES,
+        decode_block(ring + s_rpos[cur],
                      static_cast<uint32_t>((g.D + s_excl[cur]) & 15u) + my_excl, obyte, size, K.s, x);
         if (tid == 0) bulk_wait_read0();  // the previous tile's store has read ostage
         __syncthreads();
+        if (tid == 0 && deferred) {  // the ring is empty now: fetch the next payload
+            launch(nraw_p, nraw_i, cur ^ 1, true);
+            pending = true;
+        }
         const bool full = b < g.nfull;
         if (full) {
             store_block(ostage, tid, x);
