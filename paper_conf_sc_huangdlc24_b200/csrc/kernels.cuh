@@ -587,36 +587,34 @@ struct HdrStatic {
     uint32_t flags;    // CSZP2_FLAG_* (ablations)
 };
 
-// Warp-specialised compression CTA (NT_COMP = 384 threads = 12 warps):
-//   producers  warps 0-7   one thread per 32-value block: take a loaded tile, read it
-//                          into registers (freeing its TMA buffer at once), encode it
-//                          (❶ ❷), publish its aggregate, stage its payload in a
-//                          byte ring, queue it;
-//   loader     warp 8      claims tiles from the atomic ticket and TMA-loads them into
-//                          two input buffers, one tile ahead of the producers;
-//   resolver   warp 9      decoupled lookback (❸) of the queued tiles, in order (a
-//                          second resolver warp starts lookbacks before their
-//                          predecessors are published and measured slower);
-//   writers    warps 10-11 copy each resolved payload out of the ring to its place
-//                          (❹), in order, then free its ring bytes and queue slot.
-// Input buffers are released as soon as the producers hold the values, and the
-// (small, at useful compression ratios) payloads wait for their prefix in the ring,
-// so neither the loads nor the producers ever wait behind a lookback: a claimed
-// tile's aggregate appears within one load + encode of the claim.
-constexpr int NT_COMP = NT + 128;
-constexpr int LOADER_WARP = NT / 32;       // warp 8
-constexpr int RESOLVE_WARP = NT / 32 + 1;  // warp 9
-constexpr int NRESOLVE = 1;                // lookback warps (queue entries round-robin)
-constexpr int WRITER0 = NT + 64;           // first writer thread (warps 10-11)
-constexpr int NWRITER = NT_COMP - WRITER0; // 64 writer threads
-constexpr int NQ = 16;                     // queue slots (tiles staged ahead of the writers)
-constexpr uint32_t BAR_PROD = 1, BAR_WRITE = 2;
+// Warp-specialised compression CTA (NT_COMP = 288 threads = 9 warps; 3 CTAs per SM
+// for f32):
+//   producers  warps 0-7  one thread per 32-value block. Thread 0 also claims
+//                         tiles from the atomic ticket (in order, so every predecessor a
+//                         lookback waits for belongs to a running CTA) and TMA-loads
+//                         them, one tile ahead, into the single input buffer, which is
+//                         free again as soon as the values are in registers. Per tile:
+//                         encode (❶ ❷), publish the aggregate, stage the payload in a
+//                         byte ring, queue it.
+//   resolver   warp 8     for each queued tile, in order: decoupled lookback (❸), then
+//                         copy its payload from the ring to its place (❹) and free the
+//                         ring bytes and the queue slot; the last tile also writes
+//                         pads, header and *d_out_bytes.
+// The rule that keeps the GPU from serialising on the inclusive-prefix frontier: a
+// claimed tile never waits on anything that depends on a lookback. The next tile is
+// claimed ahead only while the ring clearly has room for two more payloads (so the
+// producers do not block on the ring while holding it); otherwise it is claimed after
+// the current tile is staged.
+constexpr int NT_COMP = NT + 32;
+constexpr int RESOLVE_WARP = NT / 32;  // warp 8
+constexpr int NQ = 16;                 // queue slots (tiles staged ahead of the resolver)
+constexpr uint32_t BAR_PROD = 1;
 
 template <typename T>
 struct CompLayout {
     static constexpr uint32_t IN_BYTES = Traits<T>::TILE_BYTES;  // one TMA tile
-    static constexpr uint32_t RING = sizeof(T) == 4 ? 40960u : 36864u;  // >= one max payload
-    static constexpr int SMEM = 2 * IN_BYTES + RING + 64 + 1024;
+    static constexpr uint32_t RING = 33792;                      // > one max payload
+    static constexpr int SMEM = IN_BYTES + RING + 64 + 1024;
 };
 template <typename T>
 constexpr int compress_smem_bytes() {
@@ -626,7 +624,7 @@ constexpr int compress_smem_bytes() {
 // Copy a tile's staged payload (smem, 16-byte aligned base) to its global byte
 // range [dst0, dst0 + bytes) with threads w = 0..nw-1: 16-byte aligned chunks by
 // coalesced 128-bit stores (funnel-shifted out of smem), the unaligned head/tail by
-// bytes.
+// bytes (nw >= 32).
 __device__ __forceinline__ void write_payload(const uint8_t *stg, uint8_t *out, uint64_t dst0,
                                               uint32_t bytes, int w, int nw) {
     const uint64_t dst1 = dst0 + bytes;
@@ -660,7 +658,7 @@ __device__ __forceinline__ void write_payload(const uint8_t *stg, uint8_t *out, 
 }
 
 template <typename T, bool OUTLIER>
-__global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kernel(
+__global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kernel(
     const __grid_constant__ CUtensorMap tmap, const T *__restrict__ in, const Geom g,
     const double eb_abs_arg, const int eb_from_header, uint8_t *__restrict__ out,
     unsigned *__restrict__ ticket, uint64_t *__restrict__ d_out_bytes, const HdrStatic hs) {
@@ -668,69 +666,83 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
     extern __shared__ uint8_t smem_raw[];
     uint8_t *inbuf = reinterpret_cast<uint8_t *>(
         (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    uint8_t *ring = inbuf + 2 * LY::IN_BYTES;
-    __shared__ uint64_t s_full[2], s_free[2];                      // input buffers
-    __shared__ uint64_t s_staged[NQ], s_resolved[NQ], s_done[NQ];  // queue slots
-    __shared__ uint32_t s_tkin[2];
-    __shared__ uint64_t s_qt[NQ], s_qexcl[NQ];
+    uint8_t *ring = inbuf + LY::IN_BYTES;
+    __shared__ uint64_t s_full;                    // input buffer
+    __shared__ uint64_t s_staged[NQ], s_done[NQ];  // queue slots
+    __shared__ uint64_t s_qt[NQ];
     __shared__ uint32_t s_qagg[NQ], s_qpos[NQ];
-    __shared__ uint8_t s_qbad[NQ], s_qrng[NQ];
+    __shared__ uint8_t s_qbad[NQ];
     __shared__ uint32_t s_warp[NT / 32];
-    __shared__ uint32_t s_pos;
-    __shared__ volatile uint32_t s_tail;  // ring bytes released by the writers
-    __shared__ volatile uint32_t s_head;  // ring bytes allocated by the producers
-    __shared__ volatile uint32_t s_last_agg;  // payload bytes of the latest tile
-    __shared__ volatile uint32_t s_alloc_it;  // producer iterations holding ring space
+    __shared__ uint32_t s_pos, s_tkin;
+    __shared__ volatile uint32_t s_tail;  // ring bytes released by the resolver
     __shared__ volatile uint32_t s_end;   // queue index of the end marker
 
     const int tid = threadIdx.x;
     const int warp = tid >> 5;
     const uint64_t T_eff = g.T ? g.T : 1;
     uint64_t *index = reinterpret_cast<uint64_t *>(out + 64);
+    const double eb_abs =
+        eb_from_header ? *reinterpret_cast<const volatile double *>(out + 32) : eb_abs_arg;
+
+    // producer thread 0: TMA-load tile tk into the input buffer (always arrives on
+    // s_full so its phase advances even without data)
+    auto issue = [&](uint64_t tk) {
+        const uint64_t b0 = tk * BPT;
+        if (b0 < g.nfull) {
+            if (Traits<T>::ROWS == 1) {
+                mbar_expect_tx(&s_full, BPT * 128);
+                tma_load_2d(inbuf, &tmap, 0, static_cast<int>(b0), &s_full);
+            } else {
+                const bool second = (b0 + BPT / 2) < g.nfull;
+                mbar_expect_tx(&s_full, second ? 2 * BPT * 128 : BPT * 128);
+                tma_load_2d(inbuf, &tmap, 0, static_cast<int>(2 * b0), &s_full);
+                if (second) tma_load_2d(inbuf + BPT * 128, &tmap, 0, static_cast<int>(2 * b0 + BPT), &s_full);
+            }
+        } else {
+            mbar_expect_tx(&s_full, 0);
+        }
+    };
 
     if (tid == 0) {
         s_end = 0xFFFFFFFFu;
         s_tail = 0;
-        s_head = 0;
-        s_last_agg = 0;
-        s_alloc_it = 0;
-        for (int i = 0; i < 2; i++) {
-            mbar_init(&s_full[i], 1);
-            mbar_init(&s_free[i], 1);
-        }
+        mbar_init(&s_full, 1);
         for (int i = 0; i < NQ; i++) {
             mbar_init(&s_staged[i], 1);
-            mbar_init(&s_resolved[i], 1);
             mbar_init(&s_done[i], 1);
         }
         fence_mbar_init();
+        const uint32_t tk = atomicAdd(ticket, 1u);
+        s_tkin = tk;
+        if (tk < T_eff) {
+            TRACE(tk, 0, gtimer());
+            TRACE(tk, 7, blockIdx.x);
+            issue(tk);
+        }
     }
     __syncthreads();
 
-    if (warp < LOADER_WARP) {
+    if (warp < RESOLVE_WARP) {
         // ============================== producers
-        const double eb_abs =
-            eb_from_header ? *reinterpret_cast<const volatile double *>(out + 32) : eb_abs_arg;
         const auto K = make_consts(eb_abs, static_cast<T *>(nullptr));
-        uint32_t head = 0;  // ring allocation cursor (thread 0)
+        uint32_t head = 0, last_agg = 0;  // ring allocation cursor, latest payload (thread 0)
         for (uint32_t it = 0;; ++it) {
-            const int bi = it & 1;
             const int q = it % NQ;
-            mbar_wait(&s_full[bi], (it >> 1) & 1);
-            const uint64_t t = s_tkin[bi];
-            if (t >= T_eff) {  // end marker for the resolver and the writers
+            const uint64_t t = s_tkin;  // visible: barrier at the end of the previous iteration
+            if (t >= T_eff) {           // end marker for the resolver
                 if (tid == 0) {
-                    for (int j = 0; j < NRESOLVE; j++) {  // release every resolver's pending wait
-                        const uint32_t ij = it + j;
-                        if (ij >= NQ) mbar_wait(&s_done[ij % NQ], (ij / NQ - 1) & 1);
-                    }
+                    if (it >= NQ) mbar_wait(&s_done[q], (it / NQ - 1) & 1);
                     s_end = it;
-                    for (int j = 0; j < NRESOLVE; j++) mbar_arrive(&s_staged[(it + j) % NQ]);
+                    mbar_arrive(&s_staged[q]);
                 }
                 break;
             }
+            // claim the next tile now if the ring clearly has room for two more payloads
+            uint32_t tk_next = 0;
+            const bool ahead = (tid == 0) && (head - s_tail + 2 * last_agg + 64 <= LY::RING);
+            if (ahead) tk_next = atomicAdd(ticket, 1u);  // consumed after the buffer is free
+            mbar_wait(&s_full, it & 1);
             if (tid == 0) TRACE(t, 1, gtimer());
-            const uint8_t *tile = inbuf + bi * LY::IN_BYTES;
             const uint64_t b = t * BPT + tid;
             const bool active = b < g.nb;
             const bool full = b < g.nfull;
@@ -738,7 +750,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
             T x[L];
             uint32_t valid = L;
             if (full) {
-                load_block(tile, tid, x);
+                load_block(inbuf, tid, x);
             } else {
                 valid = active ? static_cast<uint32_t>(g.n - b * L) : 0u;
 #pragma unroll
@@ -787,9 +799,17 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
             }
             if (!K.ok) bad = true;
 
-            // intra-tile scan ("Reduce"); the input buffer is free after it
+            // the input buffer is free after this barrier: start the next tile's load
             const bool any_bad = named_sync_or(BAR_PROD, NT, bad);
-            if (tid == 0) mbar_arrive(&s_free[bi]);
+            if (ahead) {
+                s_tkin = tk_next;
+                if (tk_next < T_eff) {
+                    TRACE(tk_next, 0, gtimer());
+                    TRACE(tk_next, 7, blockIdx.x);
+                    issue(tk_next);
+                }
+            }
+            // intra-tile scan ("Reduce")
             uint32_t agg;
             const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg, BAR_PROD);
             if (tid == 0) {
@@ -798,11 +818,11 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
                 // ring space (16-aligned, contiguous) and a queue slot
                 uint32_t pos = (head + 15u) & ~15u;
                 if ((pos % LY::RING) + agg > LY::RING) pos = (pos / LY::RING + 1) * LY::RING;
-                while (pos + agg > s_tail + LY::RING) __nanosleep(64);
+                // wait for room; an empty ring always has room (a payload that had to skip
+                // the ring's end can then never find the skipped bytes still "in use")
+                while (pos + agg > s_tail + LY::RING && s_tail != head) __nanosleep(64);
                 head = pos + agg;
-                s_head = head;
-                s_last_agg = agg;
-                s_alloc_it = it + 1;
+                last_agg = agg;
                 if (it >= NQ) mbar_wait(&s_done[q], (it / NQ - 1) & 1);
                 s_pos = pos;
                 s_qt[q] = t;
@@ -846,107 +866,54 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
             if (tid == 0) {
                 TRACE(t, 4, gtimer());
                 mbar_arrive(&s_staged[q]);
-            }
-        }
-    } else if (warp == LOADER_WARP) {
-        // ============================== loader: claim + TMA one tile ahead
-        if ((tid & 31) == 0) {
-            for (uint32_t it = 0;; ++it) {
-                const int bi = it & 1;
-                if (it >= 2) mbar_wait_backoff(&s_free[bi], (it / 2 - 1) & 1, 100);
-                // A claimed tile must never sit behind a full ring (which drains only
-                // as lookbacks complete), or lookbacks chain up across CTAs. Claim
-                // ahead only while the ring clearly has room for the tile being encoded
-                // and this one; otherwise wait until the previous tile holds its ring
-                // space (then nothing this tile waits on depends on a lookback).
-                while (it > 0) {
-                    const uint32_t last = s_last_agg, used = s_head - s_tail;
-                    if (used + 3 * last + 64 <= LY::RING || s_alloc_it >= it) break;
-                    __nanosleep(64);
-                }
-                const uint32_t tk = atomicAdd(ticket, 1u);
-                s_tkin[bi] = tk;
-                uint64_t *bar = &s_full[bi];
-                if (tk >= T_eff) {
-                    mbar_arrive(bar);  // producers see the end
-                    break;
-                }
-                TRACE(tk, 0, gtimer());
-                TRACE(tk, 7, blockIdx.x);
-                uint8_t *dst = inbuf + bi * LY::IN_BYTES;
-                const uint64_t b0 = static_cast<uint64_t>(tk) * BPT;
-                if (b0 < g.nfull) {
-                    if (Traits<T>::ROWS == 1) {
-                        mbar_expect_tx(bar, BPT * 128);
-                        tma_load_2d(dst, &tmap, 0, static_cast<int>(b0), bar);
-                    } else {
-                        const bool second = (b0 + BPT / 2) < g.nfull;
-                        mbar_expect_tx(bar, second ? 2 * BPT * 128 : BPT * 128);
-                        tma_load_2d(dst, &tmap, 0, static_cast<int>(2 * b0), bar);
-                        if (second)
-                            tma_load_2d(dst + BPT * 128, &tmap, 0, static_cast<int>(2 * b0 + BPT), bar);
+                if (!ahead) {  // claim now, nothing unpublished held: wait for ring room first
+                    while (head - s_tail + 2 * last_agg + 64 > LY::RING && head != s_tail) __nanosleep(64);
+                    const uint32_t tk = atomicAdd(ticket, 1u);
+                    s_tkin = tk;
+                    if (tk < T_eff) {
+                        TRACE(tk, 0, gtimer());
+                        TRACE(tk, 7, blockIdx.x);
+                        issue(tk);
                     }
-                } else {
-                    mbar_expect_tx(bar, 0);
                 }
             }
+            named_sync(BAR_PROD, NT);  // s_tkin visible
         }
-    } else if (warp < RESOLVE_WARP + NRESOLVE) {
-        // ============================== resolvers: ❸, queue entry i by warp i % NRESOLVE
+    } else {
+        // ============================== resolver: ❸ then ❹, in tile order
         const int lane = tid & 31;
-        for (uint32_t it = warp - RESOLVE_WARP;; it += NRESOLVE) {
+        for (uint32_t it = 0;; ++it) {
             const int q = it % NQ;
-            mbar_wait_backoff(&s_staged[q], (it / NQ) & 1, 200);
-            if (it >= s_end) {
-                if (lane == 0 && it == s_end) mbar_arrive(&s_resolved[q]);  // writer's end
-                break;
-            }
+            mbar_wait_backoff(&s_staged[q], (it / NQ) & 1, 100);
+            if (it >= s_end) break;
             const uint64_t t = s_qt[q];
             const uint32_t agg = s_qagg[q];
+            const uint32_t pos = s_qpos[q];
             const bool bad = s_qbad[q];
             if (lane == 0) TRACE(t, 6, gtimer());
             bool rng = bad;
-            uint64_t e = 0;
+            uint64_t excl = 0;
             if (g.T && t > 0) {
                 if (hs.flags & 1u)  // ablation: plain chained scan (Fig 12 left)
-                    e = chained_prefix(index, t, agg, bad, &rng);
+                    excl = chained_prefix(index, t, agg, bad, &rng);
                 else
-                    e = lookback(index, t, agg, bad, &rng);
+                    excl = lookback(index, t, agg, bad, &rng);
             }
-            if (lane == 0) {
-                s_qexcl[q] = e;
-                s_qrng[q] = rng;
-                TRACE(t, 3, gtimer());
-                mbar_arrive(&s_resolved[q]);
-            }
-        }
-    } else {
-        // ============================== writers: ❹ payload, pads, header
-        const int w = tid - WRITER0;
-        const double eb_abs =
-            eb_from_header ? *reinterpret_cast<const volatile double *>(out + 32) : eb_abs_arg;
-        for (uint32_t it = 0;; ++it) {
-            const int q = it % NQ;
-            mbar_wait_backoff(&s_resolved[q], (it / NQ) & 1, 200);
-            if (it >= s_end) break;
-            const uint64_t t = s_qt[q];
-            const uint64_t excl = s_qexcl[q];
-            const uint32_t agg = s_qagg[q];
-            const uint32_t pos = s_qpos[q];
+            if (lane == 0) TRACE(t, 3, gtimer());
             const uint64_t dst0 = g.D + excl;
-            write_payload(ring + (pos % LY::RING), out, dst0, agg, w, NWRITER);
+            write_payload(ring + (pos % LY::RING), out, dst0, agg, lane, 32);
             if (t == T_eff - 1) {  // last tile: pads, header, d_out_bytes
                 const uint64_t dst1 = dst0 + agg;
                 __syncwarp();
-                if (w < 16) {  // zero pad after the payload
-                    const uint64_t o = dst1 + w;
+                if (lane < 16) {  // zero pad after the payload
+                    const uint64_t o = dst1 + lane;
                     if (o < roundup16(dst1)) out[o] = 0;
-                } else if (w < 32) {  // zero pad after the offset bytes
-                    const uint64_t o = g.O + g.nb + (w - 16);
+                } else {  // zero pad after the offset bytes
+                    const uint64_t o = g.O + g.nb + (lane - 16);
                     if (o < g.D) out[o] = 0;
                 }
-                if (w == 0) {
-                    const uint32_t status = s_qrng[q] ? ST_RANGE : 0u;
+                if (lane == 0) {
+                    const uint32_t status = rng ? ST_RANGE : 0u;
                     const uint64_t pb = status ? 0 : excl + agg;
                     const uint64_t total = roundup16(g.D + pb);
                     uint64_t *h = reinterpret_cast<uint64_t *>(out);
@@ -961,9 +928,9 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 2 : 1) compress_kern
                     if (d_out_bytes) *d_out_bytes = total;
                 }
             }
-            named_sync(BAR_WRITE, NWRITER);  // all writers done reading these ring bytes
-            if (w == 0) {
-                s_tail = pos + agg;  // writers go in order, so the ring frees in order
+            __syncwarp();  // every lane is done reading these ring bytes
+            if (lane == 0) {
+                s_tail = pos + agg;  // in order, so the ring frees in order
                 mbar_arrive(&s_done[q]);
             }
         }
