@@ -119,9 +119,14 @@ __device__ __forceinline__ uint32_t swz(uint32_t row, uint32_t chunk) {
     return row * 128u + ((chunk ^ (row & 7u)) << 4);
 }
 __device__ __forceinline__ void load_block(const uint8_t *tile, uint32_t r, float (&x)[L]) {
+    // row base | (r & 7) << 4 is loop-invariant; chunk c is then one XOR away
+    const uint32_t base = smem_u32(tile) + r * 128u + ((r & 7u) << 4);
 #pragma unroll
     for (int c = 0; c < 8; c++) {
-        float4 v = *reinterpret_cast<const float4 *>(tile + swz(r, c));
+        float4 v;
+        asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                     : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+                     : "r"(base ^ (static_cast<uint32_t>(c) << 4)));
         x[4 * c + 0] = v.x;
         x[4 * c + 1] = v.y;
         x[4 * c + 2] = v.z;
@@ -332,16 +337,18 @@ __device__ __forceinline__ uint32_t cta_exclusive_scan(uint32_t v, uint32_t *s_w
     }
     if (lane == 31) s_warp[warp] = inc;
     group_sync(bar_id);
-    uint32_t base = 0, tot = 0;
+    // every warp scans the NT/32 warp totals itself (3 shuffle steps)
+    constexpr int NW = NT / 32;
+    uint32_t wt = lane < NW ? s_warp[lane] : 0u;
 #pragma unroll
-    for (int w = 0; w < NT / 32; w++) {
-        uint32_t s = s_warp[w];
-        base += (w < warp) ? s : 0u;
-        tot += s;
+    for (int o = 1; o < NW; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, wt, o);
+        if (lane >= o) wt += y;
     }
-    *total = tot;
+    const uint32_t before = __shfl_sync(0xffffffffu, wt, (warp + NW - 1) % NW);
+    *total = __shfl_sync(0xffffffffu, wt, NW - 1);
     group_sync(bar_id);
-    return base + inc - v;
+    return (warp ? before : 0u) + inc - v;
 }
 
 // ❸ Decoupled lookback (Fig 13; after Merrill & Garland [25]), split
@@ -841,7 +848,9 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
                 if (OUTLIER && nob) a[0] = 0;  // the outlier slot of every plane is 0
                 const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, static_cast<unsigned>(size ? fl : 0)));
                 if (size) {
-                    if (flw <= 1) {
+                    if (flw == 0) {  // only headers (Outlier blocks with fl = 0): no planes
+                        stage_payload<0>(ring, st, sign, outl, nob, 0, a);
+                    } else if (flw <= 1) {
                         pack_planes<0>(a);
                         stage_payload<1>(ring, st, sign, outl, nob, fl, a);
                     } else if (flw <= 2) {
