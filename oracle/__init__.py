@@ -60,6 +60,10 @@ def lib():
         L.oracle_compress_ints.argtypes = [vp, u64, i32, i32, vp, pu64]
         L.oracle_decompress.argtypes = [vp, u64, vp, u64, i32]
         L.oracle_decompress_ints.argtypes = [vp, u64, vp, u64]
+        L.oracle_compress_bound_nd.argtypes = [u64, u64, u64, i32]
+        L.oracle_compress_bound_nd.restype = u64
+        L.oracle_compress_nd.argtypes = [vp, u64, u64, u64, i32, i32, dbl, i32, i32, vp, pu64]
+        L.oracle_decompress_nd.argtypes = [vp, u64, vp, u64, u64, u64, i32, i32]
         _lib = L
     return _lib
 
@@ -161,3 +165,36 @@ def decompress_ints(cmp: np.ndarray, n: int):
     q = np.zeros(n, dtype=np.int32)
     rc = lib().oracle_decompress_ints(_ptr(cmp), cmp.size, _ptr(q), n)
     return q, rc
+
+
+def compress_nd(x: np.ndarray, eb: float, eb_mode: int = ABS, enc_mode: int = OUTLIER):
+    """NEXT #3: 2D (8x8 blocks) or 3D (4x4x4) Lorenzo stream of a 2D/3D array
+    (last axis fastest). Returns (bytes, rc)."""
+    x = np.ascontiguousarray(x)
+    ndim = x.ndim
+    if ndim == 2:
+        ny, nx = x.shape
+        nz = 1
+    elif ndim == 3:
+        nz, ny, nx = x.shape
+    else:
+        raise ValueError("2D or 3D array expected")
+    out = np.zeros(lib().oracle_compress_bound_nd(nx, ny, nz, ndim), dtype=np.uint8)
+    nbytes = ctypes.c_uint64(0)
+    rc = lib().oracle_compress_nd(_ptr(x), nx, ny, nz, ndim, _dtype_code(x), eb, eb_mode, enc_mode,
+                                  _ptr(out), ctypes.byref(nbytes))
+    if rc == ERR_ARG:
+        raise ValueError("oracle_compress_nd: bad argument")
+    return out[: nbytes.value].copy(), rc
+
+
+def decompress_nd(cmp: np.ndarray, shape, dtype=np.float32):
+    cmp = np.ascontiguousarray(cmp, dtype=np.uint8)
+    out = np.zeros(int(np.prod(shape)), dtype=dtype)
+    if len(shape) == 2:
+        (ny, nx), nz = shape, 1
+    else:
+        nz, ny, nx = shape
+    rc = lib().oracle_decompress_nd(_ptr(cmp), cmp.size, _ptr(out), nx, ny, nz, len(shape),
+                                    F32 if dtype == np.float32 else F64)
+    return out.reshape(shape), rc

@@ -156,7 +156,11 @@ static int constants_ok(int dtype, double eb_abs) {
 
 /* ---------- step ❶: lossy conversion (FORMAT.md §6.3) ---------- */
 
-int oracle_quantize(const void *x, uint64_t n, int dtype, double eb_abs, int32_t *q) {
+/* FORMAT.md §6.3 / §7: largest accepted |t| per predictor (1D, 2D, 3D) */
+static const float TMAX_F32[3] = {1073741760.0f, 268435440.0f, 134217720.0f};
+static const double TMAX_F64[3] = {1073741823.0, 268435455.0, 134217727.0};
+
+static int quantize_p(const void *x, uint64_t n, int dtype, double eb_abs, int32_t *q, int pred) {
     int status = ORC_OK;
     if (!constants_ok(dtype, eb_abs)) status = ORC_ERR_RANGE;
     if (dtype == ORC_F32) {
@@ -164,7 +168,7 @@ int oracle_quantize(const void *x, uint64_t n, int dtype, double eb_abs, int32_t
         float inv = (float)(1.0 / (2.0 * eb_abs));
         for (uint64_t i = 0; i < n; i++) {
             float t = v[i] * inv; /* one RN multiply in f32 */
-            if (!(fabsf(t) <= 1073741760.0f)) {
+            if (!(fabsf(t) <= TMAX_F32[pred])) {
                 status = ORC_ERR_RANGE;
                 q[i] = 0;
                 continue;
@@ -176,7 +180,7 @@ int oracle_quantize(const void *x, uint64_t n, int dtype, double eb_abs, int32_t
         double inv = 1.0 / (2.0 * eb_abs);
         for (uint64_t i = 0; i < n; i++) {
             double t = v[i] * inv;
-            if (!(fabs(t) <= 1073741823.0)) {
+            if (!(fabs(t) <= TMAX_F64[pred])) {
                 status = ORC_ERR_RANGE;
                 q[i] = 0;
                 continue;
@@ -185,6 +189,10 @@ int oracle_quantize(const void *x, uint64_t n, int dtype, double eb_abs, int32_t
         }
     }
     return status;
+}
+
+int oracle_quantize(const void *x, uint64_t n, int dtype, double eb_abs, int32_t *q) {
+    return quantize_p(x, n, dtype, eb_abs, q, 0);
 }
 
 void oracle_dequantize(const int32_t *q, uint64_t n, int dtype, double eb_abs, void *x) {
@@ -201,18 +209,13 @@ void oracle_dequantize(const int32_t *q, uint64_t n, int dtype, double eb_abs, v
 
 /* ---------- step ❷: first-order difference + FLE ---------- */
 
-int oracle_encode_block(const int32_t *q, int L, int enc_mode, uint8_t *offset_byte,
-                        uint8_t *payload) {
-    int32_t d[64];
+/* ❷ FLE of one block of L residuals d: offset byte + payload; returns
+ * the payload size. */
+static int fle_encode(const int32_t *d, int L, int enc_mode, uint8_t *offset_byte,
+                      uint8_t *payload) {
     uint32_t a[64];
     int fb = L / 8; /* bytes per bit field */
-
-    /* first-order difference inside the block, q_{-1} = 0 (P:130, FORMAT.md §6.4) */
-    for (int i = 0; i < L; i++) {
-        int32_t prev = (i == 0) ? 0 : q[i - 1];
-        d[i] = (int32_t)((int64_t)q[i] - (int64_t)prev);
-        a[i] = (uint32_t)(d[i] < 0 ? -(int64_t)d[i] : (int64_t)d[i]);
-    }
+    for (int i = 0; i < L; i++) a[i] = (uint32_t)(d[i] < 0 ? -(int64_t)d[i] : (int64_t)d[i]);
 
     /* Plain-FLE statistics */
     uint32_t or_all = 0;
@@ -263,6 +266,17 @@ int oracle_encode_block(const int32_t *q, int L, int enc_mode, uint8_t *offset_b
     return size_o;
 }
 
+int oracle_encode_block(const int32_t *q, int L, int enc_mode, uint8_t *offset_byte,
+                        uint8_t *payload) {
+    int32_t d[64];
+    /* first-order difference inside the block, q_{-1} = 0 (P:130, FORMAT.md §6.4) */
+    for (int i = 0; i < L; i++) {
+        int32_t prev = (i == 0) ? 0 : q[i - 1];
+        d[i] = (int32_t)((int64_t)q[i] - (int64_t)prev);
+    }
+    return fle_encode(d, L, enc_mode, offset_byte, payload);
+}
+
 int oracle_block_size(uint8_t ob_byte, int L) {
     int fb = L / 8;
     int fl = ob_byte & 31;
@@ -274,12 +288,12 @@ int oracle_block_size(uint8_t ob_byte, int L) {
     return fl ? fb * (1 + fl) : 0;
 }
 
-int oracle_decode_block(uint8_t ob_byte, const uint8_t *payload, int L, int32_t *q) {
+/* ❷⁻¹: residuals of one block from its offset byte + payload (size or -1) */
+static int fle_decode(uint8_t ob_byte, const uint8_t *payload, int L, int32_t *d) {
     int fb = L / 8;
     int size = oracle_block_size(ob_byte, L);
     if (size < 0) return -1;
     uint32_t a[64];
-    int32_t d[64];
     for (int i = 0; i < L; i++) a[i] = 0;
     int fl = ob_byte & 31;
     if (size > 0) {
@@ -304,6 +318,13 @@ int oracle_decode_block(uint8_t ob_byte, const uint8_t *payload, int L, int32_t 
     } else {
         for (int i = 0; i < L; i++) d[i] = 0;
     }
+    return size;
+}
+
+int oracle_decode_block(uint8_t ob_byte, const uint8_t *payload, int L, int32_t *q) {
+    int32_t d[64];
+    int size = fle_decode(ob_byte, payload, L, d);
+    if (size < 0) return -1;
     /* inverse first-order difference, q_{-1} = 0 (FORMAT.md §6.6) */
     int32_t prev = 0;
     for (int i = 0; i < L; i++) {
@@ -421,6 +442,7 @@ static int decode_stream(const uint8_t *cmp, uint64_t cmp_bytes, uint64_t n, int
     int L = 1 << log2L;
     *L_out = L;
     if (get_u16(cmp + 10) != BPT) return ORC_ERR_FORMAT;
+    if (cmp[12] != 0) return ORC_ERR_FORMAT; /* a multi-dimensional stream (FORMAT.md §7) */
     if (get_u64(cmp + 16) != n) return ORC_ERR_FORMAT;
     if (cmp[9] == ORC_ERR_RANGE) return ORC_ERR_RANGE;
     if (cmp[9] != 0) return ORC_ERR_FORMAT;
@@ -465,4 +487,170 @@ int oracle_decompress(const uint8_t *cmp, uint64_t cmp_bytes, void *out, uint64_
 int oracle_decompress_ints(const uint8_t *cmp, uint64_t cmp_bytes, int32_t *q, uint64_t n) {
     int L = 32;
     return decode_stream(cmp, cmp_bytes, n, q, &L);
+}
+
+/* ---------- NEXT #3: multi-dimensional Lorenzo (Table VI; FORMAT.md §7) ---------- */
+
+typedef struct {
+    uint64_t nx, ny, nz;  /* field extents, x fastest */
+    int ndim, bx, by, bz; /* block shape: 8x8 (2D) or 4x4x4 (3D), 64 values */
+    uint64_t nbx, nby, nbz, nb;
+} ndgeom_t;
+
+static int nd_setup(ndgeom_t *g, uint64_t nx, uint64_t ny, uint64_t nz, int ndim) {
+    if (ndim != 2 && ndim != 3) return ORC_ERR_ARG;
+    if (ndim == 2) nz = 1;
+    g->nx = nx;
+    g->ny = ny;
+    g->nz = nz;
+    g->ndim = ndim;
+    g->bx = g->by = (ndim == 2) ? 8 : 4;
+    g->bz = (ndim == 2) ? 1 : 4;
+    g->nbx = (nx + g->bx - 1) / g->bx;
+    g->nby = (ny + g->by - 1) / g->by;
+    g->nbz = (nz + g->bz - 1) / g->bz;
+    g->nb = g->nbx * g->nby * g->nbz;
+    return ORC_OK;
+}
+
+/* field linear index of value i (x fastest inside the block) of block b (blocks in
+ * x-fastest order over the block grid), or -1 outside the field */
+static int64_t nd_index(const ndgeom_t *g, uint64_t b, int i) {
+    uint64_t cbx = b % g->nbx, cby = (b / g->nbx) % g->nby, cbz = b / (g->nbx * g->nby);
+    int ix = i % g->bx, iy = (i / g->bx) % g->by, iz = i / (g->bx * g->by);
+    uint64_t x = cbx * g->bx + ix, y = cby * g->by + iy, z = cbz * g->bz + iz;
+    if (x >= g->nx || y >= g->ny || z >= g->nz) return -1;
+    return (int64_t)((z * g->ny + y) * g->nx + x);
+}
+
+/* q at in-block (ix, iy, iz); 0 outside the block (block-local prediction, like q_-1) */
+static int64_t qat(const int32_t *q, const ndgeom_t *g, int ix, int iy, int iz) {
+    if (ix < 0 || iy < 0 || iz < 0) return 0;
+    return q[(iz * g->by + iy) * g->bx + ix];
+}
+
+/* Lorenzo prediction of value (ix, iy, iz) from its 3 (2D) / 7 (3D) lower neighbours
+ * ("2D and 3D processing involve calculations with 3 and 7 adjacent data points") */
+static int64_t lorenzo_pred(const int32_t *q, const ndgeom_t *g, int ix, int iy, int iz) {
+    if (g->ndim == 2)
+        return qat(q, g, ix - 1, iy, 0) + qat(q, g, ix, iy - 1, 0) - qat(q, g, ix - 1, iy - 1, 0);
+    return qat(q, g, ix - 1, iy, iz) + qat(q, g, ix, iy - 1, iz) + qat(q, g, ix, iy, iz - 1) -
+           qat(q, g, ix - 1, iy - 1, iz) - qat(q, g, ix - 1, iy, iz - 1) -
+           qat(q, g, ix, iy - 1, iz - 1) + qat(q, g, ix - 1, iy - 1, iz - 1);
+}
+
+uint64_t oracle_compress_bound_nd(uint64_t nx, uint64_t ny, uint64_t nz, int ndim) {
+    ndgeom_t g;
+    if (nd_setup(&g, nx, ny, nz, ndim)) return 0;
+    uint64_t T = (g.nb + BPT - 1) / BPT;
+    uint64_t O = roundup16(64 + 8 * T), D = roundup16(O + g.nb);
+    return roundup16(D + 4 * 64 * g.nb);
+}
+
+int oracle_compress_nd(const void *x, uint64_t nx, uint64_t ny, uint64_t nz, int ndim,
+                       int dtype, double eb, int eb_mode, int enc_mode, uint8_t *out,
+                       uint64_t *out_bytes) {
+    ndgeom_t g;
+    if (nd_setup(&g, nx, ny, nz, ndim) || (dtype != ORC_F32 && dtype != ORC_F64) ||
+        (enc_mode != ORC_PLAIN && enc_mode != ORC_OUTLIER) || nx >= (1ull << 32) ||
+        ny >= (1ull << 32))
+        return ORC_ERR_ARG;
+    uint64_t n = g.nx * g.ny * g.nz;
+    if (!x && n) return ORC_ERR_ARG;
+    double eb_abs = 0.0;
+    int rc = oracle_resolve_eb(x, n, dtype, eb, eb_mode, &eb_abs);
+    if (rc != ORC_OK) return rc;
+    int32_t *q = (int32_t *)malloc((size_t)(n ? n : 1) * sizeof(int32_t));
+    if (!q) return ORC_ERR_ARG;
+    /* ❶ with the tighter range of this predictor (|d| <= 2^ndim * max|q|) */
+    int status = quantize_p(x, n, dtype, eb_abs, q, ndim - 1);
+
+    uint64_t T = (g.nb + BPT - 1) / BPT;
+    uint64_t O = roundup16(64 + 8 * T), D = roundup16(O + g.nb);
+    uint64_t excl = 0, total;
+    if (status == ORC_OK) {
+        memset(out, 0, (size_t)D);
+        int32_t blk[64], d[64];
+        int valid[64];
+        uint8_t buf[4 * 64 + 8];
+        for (uint64_t b = 0; b < g.nb; b++) {
+            for (int i = 0; i < 64; i++) {
+                int64_t idx = nd_index(&g, b, i);
+                valid[i] = idx >= 0;
+                blk[i] = valid[i] ? q[idx] : 0;
+            }
+            /* residuals: value minus its Lorenzo prediction; 0 outside the field */
+            for (int i = 0; i < 64; i++) {
+                int ix = i % g.bx, iy = (i / g.bx) % g.by, iz = i / (g.bx * g.by);
+                d[i] = valid[i] ? (int32_t)(blk[i] - lorenzo_pred(blk, &g, ix, iy, iz)) : 0;
+            }
+            uint8_t ob_byte = 0;
+            int size = fle_encode(d, 64, enc_mode, &ob_byte, buf);
+            out[O + b] = ob_byte;
+            memcpy(out + D + excl, buf, (size_t)size);
+            excl += (uint64_t)size;
+            if ((b + 1) % BPT == 0 || b + 1 == g.nb) put_u64(out + 64 + 8 * (b / BPT), (2ull << 62) | excl);
+        }
+        total = roundup16(D + excl);
+        memset(out + D + excl, 0, (size_t)(total - D - excl));
+    } else {
+        excl = 0;
+        total = roundup16(D);
+        memset(out, 0, (size_t)total);
+    }
+    free(q);
+    write_header(out, dtype, enc_mode, 64, eb_mode, status, n, eb, eb_abs, excl, total);
+    out[12] = (uint8_t)(ndim - 1);
+    put_u32(out + 56, (uint32_t)g.nx);
+    put_u32(out + 60, (uint32_t)g.ny);
+    *out_bytes = total;
+    return status;
+}
+
+int oracle_decompress_nd(const uint8_t *cmp, uint64_t cmp_bytes, void *out, uint64_t nx,
+                         uint64_t ny, uint64_t nz, int ndim, int dtype) {
+    ndgeom_t g;
+    if (nd_setup(&g, nx, ny, nz, ndim)) return ORC_ERR_ARG;
+    uint64_t n = g.nx * g.ny * g.nz;
+    if (cmp_bytes < 64 || get_u32(cmp) != MAGIC || cmp[4] != 1 || cmp[5] != (uint8_t)dtype ||
+        cmp[7] != 6 || cmp[12] != (uint8_t)(ndim - 1) || get_u16(cmp + 10) != BPT ||
+        get_u64(cmp + 16) != n || get_u32(cmp + 56) != (uint32_t)g.nx ||
+        get_u32(cmp + 60) != (uint32_t)g.ny)
+        return ORC_ERR_FORMAT;
+    if (cmp[9] == ORC_ERR_RANGE) return ORC_ERR_RANGE;
+    if (cmp[9] != 0) return ORC_ERR_FORMAT;
+    uint64_t T = (g.nb + BPT - 1) / BPT;
+    uint64_t O = roundup16(64 + 8 * T), D = roundup16(O + g.nb);
+    uint64_t pb = get_u64(cmp + 40), total = get_u64(cmp + 48);
+    if (total != roundup16(D + pb) || total > cmp_bytes) return ORC_ERR_FORMAT;
+    int32_t *q = (int32_t *)malloc((size_t)(n ? n : 1) * sizeof(int32_t));
+    if (!q) return ORC_ERR_ARG;
+    uint64_t excl = 0;
+    int32_t d[64], blk[64];
+    int rc = ORC_OK;
+    for (uint64_t b = 0; b < g.nb && rc == ORC_OK; b++) {
+        int size = oracle_block_size(cmp[O + b], 64);
+        if (size < 0 || excl + (uint64_t)size > pb) {
+            rc = ORC_ERR_FORMAT;
+            break;
+        }
+        fle_decode(cmp[O + b], cmp + D + excl, 64, d);
+        excl += (uint64_t)size;
+        /* inverse Lorenzo in index order: value = residual + prediction */
+        for (int i = 0; i < 64; i++) {
+            int ix = i % g.bx, iy = (i / g.bx) % g.by, iz = i / (g.bx * g.by);
+            blk[i] = (int32_t)((int64_t)d[i] + lorenzo_pred(blk, &g, ix, iy, iz));
+        }
+        for (int i = 0; i < 64; i++) {
+            int64_t idx = nd_index(&g, b, i);
+            if (idx >= 0) q[idx] = blk[i];
+        }
+        if (((b + 1) % BPT == 0 || b + 1 == g.nb) &&
+            get_u64(cmp + 64 + 8 * (b / BPT)) != ((2ull << 62) | excl))
+            rc = ORC_ERR_FORMAT;
+    }
+    if (rc == ORC_OK && excl != pb) rc = ORC_ERR_FORMAT;
+    if (rc == ORC_OK) oracle_dequantize(q, n, dtype, get_f64(cmp + 32), out);
+    free(q);
+    return rc;
 }

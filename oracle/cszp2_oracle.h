@@ -75,4 +75,13 @@ int oracle_decompress(const uint8_t *cmp, uint64_t cmp_bytes, void *out, uint64_
 /* Lossless inverse of oracle_compress_ints. */
 int oracle_decompress_ints(const uint8_t *cmp, uint64_t cmp_bytes, int32_t *q, uint64_t n);
 
+/* NEXT #3 (Table VI; FORMAT.md §7): 2D Lorenzo on 8x8 blocks / 3D Lorenzo on
+ * 4x4x4 blocks of an nx x ny (x nz) field (x fastest), L = 64, same FLE. */
+uint64_t oracle_compress_bound_nd(uint64_t nx, uint64_t ny, uint64_t nz, int ndim);
+int oracle_compress_nd(const void *x, uint64_t nx, uint64_t ny, uint64_t nz, int ndim,
+                       int dtype, double eb, int eb_mode, int enc_mode, uint8_t *out,
+                       uint64_t *out_bytes);
+int oracle_decompress_nd(const uint8_t *cmp, uint64_t cmp_bytes, void *out, uint64_t nx,
+                         uint64_t ny, uint64_t nz, int ndim, int dtype);
+
 #endif
