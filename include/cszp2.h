@@ -147,6 +147,30 @@ int cszp2_decompress_host(const void *h_cmp, uint64_t cmp_bytes, void *d_cmp_wor
 int cszp2_container_index(const uint64_t *d_sizes, int nparts, uint64_t *d_offsets,
                           void *stream);
 
+/* ---- Multi-dimensional Lorenzo layouts (§VI-D,
+ * Table VI; FORMAT.md §7). The paper's 2D (8x8 block) and 3D (4x4x4 block)
+ * variants of the same single-kernel design: L = 64 values per block, residual =
+ * value − Lorenzo prediction from the 3 (2D) / 7 (3D) lower in-block neighbours
+ * (neighbours outside the block are 0), then the same Plain/Outlier FLE (8-byte
+ * bit fields) and decoupled-lookback concatenation. The stream carries predictor
+ * id and nx, ny in its header (a 1D decoder refuses it, and vice versa).
+ *  field      : nx * ny (* nz) values of `dtype`, row-major with x fastest,
+ *               device, 16-byte aligned. ndim = 2 requires nz = 1.
+ *  extents    : nx, ny, nz < 2^32 and nx*ny*nz <= 2^40, else ARG.
+ * cszp2_compress_bound_nd: bytes d_out must hold (0 on bad arguments), including
+ *   16 bytes of scratch past the stream, as cszp2_compress_bound.
+ * cszp2_compress_nd: like cszp2_compress (same eb / eb_mode / enc_mode meaning,
+ *   same RANGE behaviour with this predictor's tighter limit |x/2eb| <= 2^28-1 (2D)
+ *   or 2^27-1 (3D), FORMAT.md §7); asynchronous on `stream`.
+ * cszp2_decompress_nd: inverse; d_out = nx*ny*nz values (any 4/8-byte alignment);
+ *   d_status as in cszp2_decompress. */
+uint64_t cszp2_compress_bound_nd(uint64_t nx, uint64_t ny, uint64_t nz, int ndim, int dtype);
+int cszp2_compress_nd(const void *d_in, uint64_t nx, uint64_t ny, uint64_t nz, int ndim, int dtype,
+                      double eb, int eb_mode, int enc_mode, void *d_out, uint64_t *d_out_bytes,
+                      void *stream);
+int cszp2_decompress_nd(const void *d_cmp, void *d_out, uint64_t nx, uint64_t ny, uint64_t nz, int ndim,
+                        int dtype, int *d_status, void *stream);
+
 /* Library identification ("cszp2 <version> sm_100a"). */
 const char *cszp2_version(void);
 

@@ -68,6 +68,10 @@ def _load():
                                       ctypes.POINTER(ctypes.c_uint64), vp]
     L.cszp2_decompress_host.argtypes = [vp, u64, vp, vp, vp, u64, i32, vp, vp]
     L.cszp2_container_index.argtypes = [vp, i32, vp, vp]
+    L.cszp2_compress_bound_nd.argtypes = [u64, u64, u64, i32, i32]
+    L.cszp2_compress_bound_nd.restype = u64
+    L.cszp2_compress_nd.argtypes = [vp, u64, u64, u64, i32, i32, dbl, i32, i32, vp, vp, vp]
+    L.cszp2_decompress_nd.argtypes = [vp, vp, u64, u64, u64, i32, i32, vp, vp]
     L.cszp2_version.restype = ctypes.c_char_p
     return L
 
@@ -79,6 +83,7 @@ EXPORTED = (
     "cszp2_compress_encode_ex",
     "cszp2_decompress", "cszp2_decompress_range", "cszp2_read_header", "cszp2_compress_host", "cszp2_decompress_host",
     "cszp2_container_index", "cszp2_version",
+    "cszp2_compress_bound_nd", "cszp2_compress_nd", "cszp2_decompress_nd",
 )
 
 
@@ -211,4 +216,49 @@ def container_index(sizes: torch.Tensor, out=None, stream=None):
         out = torch.empty(sizes.numel() + 1, dtype=torch.int64, device=sizes.device)
     _check("cszp2_container_index",
            _lib.cszp2_container_index(_ptr(sizes), sizes.numel(), _ptr(out), _stream(stream)))
+    return out
+
+
+def _extents(shape):
+    """(nx, ny, nz, ndim) of a 2D (ny, nx) or 3D (nz, ny, nx) shape, x fastest."""
+    shape = tuple(int(v) for v in shape)
+    if len(shape) == 2:
+        return shape[1], shape[0], 1, 2
+    if len(shape) == 3:
+        return shape[2], shape[1], shape[0], 3
+    raise ValueError("2D or 3D field expected")
+
+
+def compress_bound_nd(shape, dtype=torch.float32) -> int:
+    nx, ny, nz, nd = _extents(shape)
+    return int(_lib.cszp2_compress_bound_nd(nx, ny, nz, nd, _DT[dtype] if isinstance(dtype, torch.dtype) else dtype))
+
+
+def compress_nd(x: torch.Tensor, eb: float, eb_mode="abs", enc_mode="outlier", out=None, out_bytes=None,
+                stream=None):
+    """2D (8x8 blocks) / 3D (4x4x4 blocks) Lorenzo compression of a 2D/3D CUDA
+    tensor (last axis fastest; FORMAT.md §7). Returns (buffer, device byte count)."""
+    _need_cuda(x, out, out_bytes)
+    x = x.contiguous()
+    nx, ny, nz, nd = _extents(x.shape)
+    dt = _DT[x.dtype]
+    if out is None:
+        out = torch.empty(compress_bound_nd(x.shape, dt), dtype=torch.uint8, device=x.device)
+    if out_bytes is None:
+        out_bytes = torch.zeros(1, dtype=torch.int64, device=x.device)
+    rc = _lib.cszp2_compress_nd(_ptr(x), nx, ny, nz, nd, dt, float(eb), _EB[eb_mode], _ENC[enc_mode],
+                                _ptr(out), _ptr(out_bytes), _stream(stream))
+    _check("cszp2_compress_nd", rc)
+    return out, out_bytes
+
+
+def decompress_nd(cmp: torch.Tensor, shape, dtype=torch.float32, out=None, status=None, stream=None):
+    """Inverse of compress_nd into a tensor of `shape`."""
+    _need_cuda(cmp, out, status)
+    nx, ny, nz, nd = _extents(shape)
+    if out is None:
+        out = torch.empty(tuple(shape), dtype=dtype, device=cmp.device)
+    rc = _lib.cszp2_decompress_nd(_ptr(cmp), _ptr(out), nx, ny, nz, nd, _DT[out.dtype], _ptr(status),
+                                  _stream(stream))
+    _check("cszp2_decompress_nd", rc)
     return out

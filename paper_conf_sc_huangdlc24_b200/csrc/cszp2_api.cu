@@ -11,6 +11,7 @@
 
 #include "cszp2.h"
 #include "kernels.cuh"
+#include "kernels_nd.cuh"
 
 using namespace cszp2;
 
@@ -169,6 +170,81 @@ int launch_decompress(const void *d_cmp, void *d_out, const Geom &g, int *d_stat
     return launch_status();
 }
 
+// ---- NEXT #3: multi-dimensional Lorenzo layouts (FORMAT.md §7)
+// 0 on success; ARG for a bad ndim / extent
+int geometry_nd(uint64_t nx, uint64_t ny, uint64_t nz, int ndim, GeomND *g) {
+    if (ndim != 2 && ndim != 3) return CSZP2_ERR_ARG;
+    if (ndim == 2) {
+        if (nz != 1) return CSZP2_ERR_ARG;
+    }
+    if (nx >= (1ull << 32) || ny >= (1ull << 32) || nz >= (1ull << 32)) return CSZP2_ERR_ARG;
+    const uint64_t b = ndim == 2 ? 8 : 4, bz = ndim == 2 ? 1 : 4;
+    g->nx = nx;
+    g->ny = ny;
+    g->nz = nz;
+    // n <= 2^40 (as 1D); checked without overflow
+    if (nx && ny && nz && (nx * ny > (1ull << 40) || nx * ny * nz / nz != nx * ny ||
+                           nx * ny * nz > (1ull << 40)))
+        return CSZP2_ERR_ARG;
+    g->n = nx * ny * nz;
+    g->nbx = (nx + b - 1) / b;
+    g->nby = (ny + b - 1) / b;
+    g->nbz = (nz + bz - 1) / bz;
+    g->nb = g->nbx * g->nby * g->nbz;
+    g->T = (g->nb + BPT - 1) / BPT;
+    g->O = roundup16(64 + 8 * g->T);
+    g->D = roundup16(g->O + g->nb);
+    return CSZP2_OK;
+}
+uint64_t stream_bound_nd(const GeomND &g) { return roundup16(g.D + static_cast<uint64_t>(4 * LND) * g.nb); }
+
+template <typename T, int NDIM, bool OUTLIER>
+int launch_compress_nd(const void *d_in, const GeomND &g, double eb, int eb_mode, int enc_mode,
+                       void *d_out, uint64_t *d_out_bytes, cudaStream_t st) {
+    static std::once_flag once;
+    static int attr_rc = CSZP2_OK;
+    constexpr int smem = ND_STAGE + 64;
+    std::call_once(once, [] { attr_rc = set_smem(compress_nd_kernel<T, NDIM, OUTLIER>, smem); });
+    if (attr_rc) return attr_rc;
+    unsigned *ticket = reinterpret_cast<unsigned *>(static_cast<uint8_t *>(d_out) + stream_bound_nd(g));
+    HdrStatic hs;
+    hs.word1 = 1u | (static_cast<uint32_t>(Traits<T>::DTYPE) << 8) |
+               (static_cast<uint32_t>(enc_mode) << 16) | (6u << 24);
+    hs.eb_mode = static_cast<uint32_t>(eb_mode);
+    hs.eb_user = eb;
+    hs.flags = 0;
+    const unsigned grid = static_cast<unsigned>(g.T ? g.T : 1);
+    compress_nd_kernel<T, NDIM, OUTLIER><<<grid, NT, smem, st>>>(
+        static_cast<const T *>(d_in), g, eb, eb_mode == CSZP2_EB_REL ? 1 : 0,
+        static_cast<uint8_t *>(d_out), ticket, d_out_bytes, hs);
+    return launch_status();
+}
+
+template <typename T, int NDIM>
+int launch_decompress_nd(const void *d_cmp, void *d_out, const GeomND &g, int *d_status,
+                         cudaStream_t st) {
+    static std::once_flag once;
+    static int attr_rc = CSZP2_OK;
+    constexpr int smem = ND_STAGE + 64;
+    std::call_once(once, [] { attr_rc = set_smem(decompress_nd_kernel<T, NDIM>, smem); });
+    if (attr_rc) return attr_rc;
+    const unsigned grid = static_cast<unsigned>(g.T ? g.T : 1);
+    decompress_nd_kernel<T, NDIM><<<grid, NT, smem, st>>>(static_cast<const uint8_t *>(d_cmp),
+                                                          static_cast<T *>(d_out), g, d_status);
+    return launch_status();
+}
+
+template <typename T>
+int dispatch_compress_nd(const void *d_in, const GeomND &g, int ndim, double eb, int eb_mode,
+                         int enc_mode, void *d_out, uint64_t *d_out_bytes, cudaStream_t st) {
+    const bool o = enc_mode == CSZP2_ENC_OUTLIER;
+    if (ndim == 2)
+        return o ? launch_compress_nd<T, 2, true>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st)
+                 : launch_compress_nd<T, 2, false>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st);
+    return o ? launch_compress_nd<T, 3, true>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st)
+             : launch_compress_nd<T, 3, false>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st);
+}
+
 }  // namespace
 
 extern "C" {
@@ -321,6 +397,47 @@ int cszp2_decompress_host(const void *h_cmp, uint64_t cmp_bytes, void *d_cmp_wor
         return CSZP2_ERR_CUDA;
     if (cudaStreamSynchronize(S(stream)) != cudaSuccess) return CSZP2_ERR_CUDA;
     return st;
+}
+
+uint64_t cszp2_compress_bound_nd(uint64_t nx, uint64_t ny, uint64_t nz, int ndim, int dtype) {
+    GeomND g;
+    if (!wsize(dtype) || geometry_nd(nx, ny, nz, ndim, &g)) return 0;
+    return stream_bound_nd(g) + 16;  // + the ticket scratch, as cszp2_compress_bound
+}
+
+int cszp2_compress_nd(const void *d_in, uint64_t nx, uint64_t ny, uint64_t nz, int ndim, int dtype,
+                      double eb, int eb_mode, int enc_mode, void *d_out, uint64_t *d_out_bytes,
+                      void *stream) {
+    GeomND g;
+    if (geometry_nd(nx, ny, nz, ndim, &g)) return CSZP2_ERR_ARG;
+    if (enc_mode != CSZP2_ENC_PLAIN && enc_mode != CSZP2_ENC_OUTLIER) return CSZP2_ERR_ARG;
+    int rc = check_compress_args(d_in, g.n, dtype, eb, eb_mode, d_out);
+    if (rc) return rc;
+    cudaStream_t st = S(stream);
+    if (cudaMemsetAsync(d_out, 0, g.O, st) != cudaSuccess ||
+        cudaMemsetAsync(static_cast<uint8_t *>(d_out) + stream_bound_nd(g), 0, 16, st) != cudaSuccess)
+        return CSZP2_ERR_CUDA;
+    if (eb_mode == CSZP2_EB_REL) {
+        rc = dtype == CSZP2_F32 ? launch_minmax<float>(d_in, g.n, eb, d_out, st)
+                                : launch_minmax<double>(d_in, g.n, eb, d_out, st);
+        if (rc) return rc;
+    }
+    return dtype == CSZP2_F32
+               ? dispatch_compress_nd<float>(d_in, g, ndim, eb, eb_mode, enc_mode, d_out, d_out_bytes, st)
+               : dispatch_compress_nd<double>(d_in, g, ndim, eb, eb_mode, enc_mode, d_out, d_out_bytes, st);
+}
+
+int cszp2_decompress_nd(const void *d_cmp, void *d_out, uint64_t nx, uint64_t ny, uint64_t nz, int ndim,
+                        int dtype, int *d_status, void *stream) {
+    GeomND g;
+    if (!wsize(dtype) || !d_cmp || geometry_nd(nx, ny, nz, ndim, &g)) return CSZP2_ERR_ARG;
+    if ((!d_out && g.n) || !aligned16(d_cmp)) return CSZP2_ERR_ARG;
+    cudaStream_t st = S(stream);
+    if (dtype == CSZP2_F32)
+        return ndim == 2 ? launch_decompress_nd<float, 2>(d_cmp, d_out, g, d_status, st)
+                         : launch_decompress_nd<float, 3>(d_cmp, d_out, g, d_status, st);
+    return ndim == 2 ? launch_decompress_nd<double, 2>(d_cmp, d_out, g, d_status, st)
+                     : launch_decompress_nd<double, 3>(d_cmp, d_out, g, d_status, st);
 }
 
 int cszp2_container_index(const uint64_t *d_sizes, int nparts, uint64_t *d_offsets,

@@ -1013,7 +1013,8 @@ __device__ __forceinline__ int check_header(const uint8_t *cmp, const Geom &g, d
     int err = 0;
     const uint32_t want1 = 1u | (static_cast<uint32_t>(Traits<T>::DTYPE) << 8) | (5u << 24);
     if ((h0 & 0xFFFFFFFFu) != MAGIC || ((h0 >> 32) & 0xFF00FFFFu) != want1 ||
-        ((h1 >> 16) & 0xFFFFu) != BPT || h[2] != g.n)
+        ((h1 >> 16) & 0xFFFFu) != BPT || (h1 >> 32) != 0 /* 1D predictor, FORMAT.md §7 */ ||
+        h[2] != g.n)
         err = ST_FORMAT;
     else if (((h1 >> 8) & 0xFF) != 0)
         err = ((h1 >> 8) & 0xFF) == ST_RANGE ? ST_RANGE : ST_FORMAT;

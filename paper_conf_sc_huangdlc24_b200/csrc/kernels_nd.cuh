@@ -1,0 +1,397 @@
+// kernels_nd.cuh — NEXT #3: the multi-dimensional Lorenzo variants of the paper's
+// §VI-D / Table VI: 2D Lorenzo on 8x8 blocks and 3D Lorenzo on 4x4x4
+// blocks (L = 64), same Plain/Outlier FLE, same decoupled-lookback concatenation
+// (FORMAT.md §7). The paper keeps them out of the main design because they cost
+// throughput (>50%); these kernels favour simplicity over speed: one CTA per
+// tile (dynamic ticket), one thread per 64-value block, values gathered straight
+// from global memory.
+#pragma once
+#include "kernels.cuh"
+
+namespace cszp2 {
+
+constexpr int LND = 64;  // values per multi-dimensional block
+
+struct GeomND {
+    uint64_t nx, ny, nz;    // field extents, x fastest
+    uint64_t nbx, nby, nbz; // block grid
+    uint64_t n, nb, T, O, D;
+};
+
+template <int NDIM>
+struct BlockShape;
+template <>
+struct BlockShape<2> {
+    static constexpr int BX = 8, BY = 8, BZ = 1;
+};
+template <>
+struct BlockShape<3> {
+    static constexpr int BX = 4, BY = 4, BZ = 4;
+};
+
+// FORMAT.md §7 range limits: |d| <= 2^ndim * max|q| must fit the 31-bit code
+template <int NDIM>
+__device__ __forceinline__ int quantize_nd(float x, float inv, bool &bad) {
+    const float t = __fmul_rn(x, inv);
+    bad |= !(fabsf(t) <= (NDIM == 2 ? 268435440.0f : 134217720.0f));
+    return __float2int_rn(t);
+}
+template <int NDIM>
+__device__ __forceinline__ int quantize_nd(double x, double inv, bool &bad) {
+    const double t = __dmul_rn(x, inv);
+    bad |= !(fabs(t) <= (NDIM == 2 ? 268435455.0 : 134217727.0));
+    return __double2int_rn(t);
+}
+
+// Lorenzo prediction of in-block value i from its lower neighbours (block-local:
+// neighbours outside the block are 0), "3 and 7 adjacent data points".
+template <int NDIM>
+__device__ __forceinline__ int lorenzo_pred(const int (&q)[LND], int i) {
+    using S = BlockShape<NDIM>;
+    const int ix = i % S::BX, iy = (i / S::BX) % S::BY, iz = i / (S::BX * S::BY);
+    auto Q = [&](int dx, int dy, int dz) -> int {
+        if (ix < dx || iy < dy || iz < dz) return 0;
+        return q[i - dx - dy * S::BX - dz * S::BX * S::BY];
+    };
+    if (NDIM == 2) return Q(1, 0, 0) + Q(0, 1, 0) - Q(1, 1, 0);
+    return Q(1, 0, 0) + Q(0, 1, 0) + Q(0, 0, 1) - Q(1, 1, 0) - Q(1, 0, 1) - Q(0, 1, 1) + Q(1, 1, 1);
+}
+
+// origin (x0, y0, z0) of block b in the field
+struct BlockOrigin {
+    uint64_t x0, y0, z0;
+};
+template <int NDIM>
+__device__ __forceinline__ BlockOrigin block_origin(const GeomND &g, uint64_t b) {
+    using S = BlockShape<NDIM>;
+    BlockOrigin o;
+    const uint64_t cbx = b % g.nbx, r = b / g.nbx;
+    o.x0 = cbx * S::BX;
+    o.y0 = (r % g.nby) * S::BY;
+    o.z0 = (r / g.nby) * S::BZ;
+    return o;
+}
+// field linear index of in-block value i (compile-time after unrolling), or ~0
+// outside the field
+template <int NDIM>
+__device__ __forceinline__ uint64_t nd_index(const GeomND &g, const BlockOrigin &o, int i) {
+    using S = BlockShape<NDIM>;
+    const int ix = i % S::BX, iy = (i / S::BX) % S::BY, iz = i / (S::BX * S::BY);
+    const uint64_t x = o.x0 + ix, y = o.y0 + iy, z = o.z0 + iz;
+    if (x >= g.nx || y >= g.ny || z >= g.nz) return ~uint64_t(0);
+    return (z * g.ny + y) * g.nx + x;
+}
+
+// one 32-bit word to smem at any byte position (neighbouring blocks own the other bytes)
+__device__ __forceinline__ void put_word(uint8_t *base, uint32_t pos, uint32_t w) {
+    if ((pos & 3u) == 0) {
+        *reinterpret_cast<uint32_t *>(base + pos) = w;
+    } else {
+        for (int j = 0; j < 4; j++) base[pos + j] = static_cast<uint8_t>(w >> (8 * j));
+    }
+}
+
+constexpr uint32_t ND_STAGE = BPT * 4 * LND + 64;  // max tile payload + slack
+
+template <typename T, int NDIM, bool OUTLIER>
+__global__ void __launch_bounds__(NT) compress_nd_kernel(const T *__restrict__ in, const GeomND g,
+                                                         const double eb_abs_arg,
+                                                         const int eb_from_header,
+                                                         uint8_t *__restrict__ out,
+                                                         unsigned *__restrict__ ticket,
+                                                         uint64_t *__restrict__ d_out_bytes,
+                                                         const HdrStatic hs) {
+    extern __shared__ uint8_t stage_raw[];
+    uint8_t *stage = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(stage_raw) + 15) & ~uintptr_t(15));
+    __shared__ uint32_t s_warp[NT / 32];
+    __shared__ uint32_t s_tk;
+    __shared__ uint64_t s_excl;
+    __shared__ bool s_rng;
+    const int tid = threadIdx.x;
+    const uint64_t T_eff = g.T ? g.T : 1;
+    uint64_t *index = reinterpret_cast<uint64_t *>(out + 64);
+    if (tid == 0) s_tk = atomicAdd(ticket, 1u);  // in-order tiles: forward progress
+    __syncthreads();
+    const uint64_t t = s_tk;
+    const double eb_abs =
+        eb_from_header ? *reinterpret_cast<const volatile double *>(out + 32) : eb_abs_arg;
+    const auto K = make_consts(eb_abs, static_cast<T *>(nullptr));
+
+    const uint64_t b = t * BPT + tid;
+    const bool active = b < g.nb;
+    // ---- gather + ❶ quantize; values outside the field stay 0 and get residual 0
+    int q[LND];
+    uint64_t outside = 0;  // bit i: value i lies outside the field
+    bool bad = false;
+    const BlockOrigin bo = block_origin<NDIM>(g, active ? b : 0);
+#pragma unroll
+    for (int i = 0; i < LND; i++) {
+        const uint64_t idx = active ? nd_index<NDIM>(g, bo, i) : ~uint64_t(0);
+        q[i] = 0;
+        if (idx != ~uint64_t(0))
+            q[i] = quantize_nd<NDIM>(in[idx], K.inv, bad);
+        else
+            outside |= 1ull << i;
+    }
+    // ---- nD Lorenzo residuals, highest index first so every prediction still sees q
+    uint32_t a[LND];
+    uint64_t sign = 0;
+    uint32_t or_rest = 0;
+#pragma unroll
+    for (int i = LND - 1; i >= 0; i--) {
+        int d = q[i] - lorenzo_pred<NDIM>(q, i);
+        if ((outside >> i) & 1ull) d = 0;
+        a[i] = static_cast<uint32_t>(d < 0 ? -d : d);
+        sign |= static_cast<uint64_t>(d < 0) << i;
+        if (i) or_rest |= a[i];
+    }
+    // ---- ❷ FLE with 8-byte fields
+    const int fl_p = 32 - __clz(or_rest | a[0]);
+    uint32_t size = fl_p ? 8u * (1u + fl_p) : 0u;
+    uint32_t obyte = static_cast<uint32_t>(fl_p);
+    int fl = fl_p, nob = 0;
+    if (OUTLIER) {
+        const int fl_o = 32 - __clz(or_rest);
+        const int ob = max(1, (32 - __clz(a[0]) + 7) >> 3);
+        const uint32_t size_o = 8u + ob + 8u * fl_o;
+        if (size_o < size) {
+            size = size_o;
+            obyte = 0x80u | (static_cast<uint32_t>(ob - 1) << 5) | static_cast<uint32_t>(fl_o);
+            fl = fl_o;
+            nob = ob;
+        }
+    }
+    if (!active) {
+        size = 0;
+        bad = false;
+    }
+    if (!K.ok) bad = true;
+
+    // ---- ❸ scan + decoupled lookback
+    const bool any_bad = __syncthreads_or(bad);
+    uint32_t agg;
+    const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg);
+    if (tid < 32) {
+        bool rng = any_bad;
+        uint64_t e = 0;
+        if (g.T) {
+            if (tid == 0) publish_aggregate(index, t, agg, any_bad);
+            __syncwarp();
+            if (t > 0) e = lookback(index, t, agg, any_bad, &rng);
+        }
+        if (tid == 0) {
+            s_excl = e;
+            s_rng = rng;
+        }
+    }
+    if (active) out[g.O + b] = static_cast<uint8_t>(obyte);
+
+    // ---- payload into the stage: sign (8 B), outlier (nob B), planes (8 B each:
+    //      values 0..31 then 32..63), bit planes by two in-register transposes
+    const uint32_t outl = a[0];
+    if (OUTLIER && nob) a[0] = 0;
+    uint32_t lo[32], hi[32];
+#pragma unroll
+    for (int i = 0; i < 32; i++) {
+        lo[i] = a[i];
+        hi[i] = a[32 + i];
+    }
+    const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, static_cast<unsigned>(size ? fl : 0)));
+    if (flw > 0) {
+        if (flw <= 4) {
+            pack_planes<2>(lo);
+            pack_planes<2>(hi);
+        } else if (flw <= 8) {
+            pack_planes<3>(lo);
+            pack_planes<3>(hi);
+        } else if (flw <= 16) {
+            pack_planes<4>(lo);
+            pack_planes<4>(hi);
+        } else {
+            pack_planes<5>(lo);
+            pack_planes<5>(hi);
+        }
+    }
+    if (size) {
+        uint32_t p = my_excl;
+        put_word(stage, p, static_cast<uint32_t>(sign));
+        put_word(stage, p + 4, static_cast<uint32_t>(sign >> 32));
+        p += 8;
+        for (int j = 0; j < nob; j++) stage[p + j] = static_cast<uint8_t>(outl >> (8 * j));
+        p += nob;
+#pragma unroll
+        for (int k = 0; k < 32; k++) {
+            if (k < fl) {
+                put_word(stage, p + 8 * k, lo[k]);
+                put_word(stage, p + 8 * k + 4, hi[k]);
+            }
+        }
+    }
+    __syncthreads();  // stage complete; s_excl visible
+    const uint64_t dst0 = g.D + s_excl;
+    write_payload(stage, out, dst0, agg, tid, NT);
+    if (t == T_eff - 1) {  // last tile: pads, header, d_out_bytes
+        const uint64_t dst1 = dst0 + agg;
+        if (tid >= 32 && tid < 48) {
+            const uint64_t o = dst1 + (tid - 32);
+            if (o < roundup16(dst1)) out[o] = 0;
+        }
+        if (tid >= 64 && tid < 80) {
+            const uint64_t o = g.O + g.nb + (tid - 64);
+            if (o < g.D) out[o] = 0;
+        }
+        if (tid == 0) {
+            const uint32_t status = s_rng ? ST_RANGE : 0u;
+            const uint64_t pb = status ? 0 : s_excl + agg;
+            const uint64_t total = roundup16(g.D + pb);
+            uint64_t *h = reinterpret_cast<uint64_t *>(out);
+            h[0] = MAGIC | (static_cast<uint64_t>(hs.word1) << 32);
+            h[1] = hs.eb_mode | (status << 8) | (static_cast<uint64_t>(BPT) << 16) |
+                   (static_cast<uint64_t>(NDIM - 1) << 32);
+            h[2] = g.n;
+            h[3] = static_cast<uint64_t>(__double_as_longlong(hs.eb_user));
+            h[4] = static_cast<uint64_t>(__double_as_longlong(eb_abs));
+            h[5] = pb;
+            h[6] = total;
+            h[7] = g.nx | (g.ny << 32);
+            if (d_out_bytes) *d_out_bytes = total;
+        }
+    }
+}
+
+template <typename T, int NDIM>
+__global__ void __launch_bounds__(NT) decompress_nd_kernel(const uint8_t *__restrict__ cmp,
+                                                           T *__restrict__ out, const GeomND g,
+                                                           int *__restrict__ d_status) {
+    extern __shared__ uint8_t stage_raw[];
+    uint8_t *pbuf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(stage_raw) + 15) & ~uintptr_t(15));
+    __shared__ uint64_t s_bar;
+    __shared__ uint32_t s_warp[NT / 32];
+    __shared__ uint64_t s_excl;
+    __shared__ uint32_t s_bytes;
+    __shared__ double s_eb;
+    __shared__ int s_err;
+    const int tid = threadIdx.x;
+    const uint64_t t = blockIdx.x;
+    if (tid == 0) {
+        const uint64_t *h = reinterpret_cast<const uint64_t *>(cmp);
+        const uint64_t h0 = h[0], h1 = h[1];
+        int err = 0;
+        const uint32_t want1 = 1u | (static_cast<uint32_t>(Traits<T>::DTYPE) << 8) | (6u << 24);
+        if ((h0 & 0xFFFFFFFFu) != MAGIC || ((h0 >> 32) & 0xFF00FFFFu) != want1 ||
+            ((h1 >> 16) & 0xFFFFu) != BPT || ((h1 >> 32) & 0xFFu) != static_cast<uint64_t>(NDIM - 1) ||
+            h[2] != g.n || h[7] != (g.nx | (g.ny << 32)))
+            err = ST_FORMAT;
+        else if (((h1 >> 8) & 0xFF) != 0)
+            err = ((h1 >> 8) & 0xFF) == ST_RANGE ? ST_RANGE : ST_FORMAT;
+        const uint64_t pb = h[5];
+        if (!err && h[6] != roundup16(g.D + pb)) err = ST_FORMAT;
+        uint64_t e = 0, i = 0;
+        if (!err && t < g.T) {
+            const uint64_t *index = h + 8;
+            const uint64_t dp = t ? index[t - 1] : FLAG_P, di = index[t];
+            e = dp & VAL_MASK;
+            i = di & VAL_MASK;
+            if ((dp >> 61) != 4 || (di >> 61) != 4 || i < e || i > pb ||
+                i - e > static_cast<uint64_t>(BPT) * 4 * LND)
+                err = ST_FORMAT;
+        }
+        s_err = err;
+        s_eb = __longlong_as_double(static_cast<long long>(h[4]));
+        s_excl = e;
+        s_bytes = static_cast<uint32_t>(i - e);
+        mbar_init(&s_bar, 1);
+        fence_mbar_init();
+        if (!err && t < g.T) {
+            if (i > e) {
+                const uint64_t src0 = (g.D + e) & ~uint64_t(15);
+                const uint32_t len = static_cast<uint32_t>(roundup16(g.D + i) - src0);
+                mbar_expect_tx(&s_bar, len);
+                bulk_load(pbuf, cmp + src0, len, &s_bar);
+            } else {
+                mbar_expect_tx(&s_bar, 0);
+            }
+        }
+    }
+    __syncthreads();
+    if (s_err || t >= g.T) {
+        if (tid == 0 && s_err && d_status) atomicOr(d_status, s_err);
+        return;
+    }
+    const uint64_t b = t * BPT + tid;
+    const bool active = b < g.nb;
+    const uint32_t obyte = active ? cmp[g.O + b] : 0u;
+    const uint32_t fl = obyte & 31u;
+    const bool is_o = (obyte & 0x80u) != 0;
+    const uint32_t nob = is_o ? ((obyte >> 5) & 3u) + 1u : 0u;
+    bool bad = (!is_o && (obyte & 0x60u));
+    const uint32_t size = is_o ? 8u + nob + 8u * fl : (fl ? 8u * (1u + fl) : 0u);
+    uint32_t agg;
+    const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg);
+    bad |= (tid == 0 && agg != s_bytes);
+    const bool any_bad = __syncthreads_or(bad);
+    mbar_wait(&s_bar, 0);
+    if (any_bad) {
+        if (tid == 0 && d_status) atomicOr(d_status, ST_FORMAT);
+        return;
+    }
+    const auto K = make_consts(s_eb, static_cast<T *>(nullptr));
+    // ---- ❷⁻¹: sign (8 B), outlier, planes (8 B each) -> residual magnitudes
+    uint32_t lo[32], hi[32];
+#pragma unroll
+    for (int i = 0; i < 32; i++) lo[i] = hi[i] = 0;
+    uint64_t sign = 0;
+    uint32_t outl = 0;
+    const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, size ? fl : 0u));
+    if (size) {
+        uint32_t p = static_cast<uint32_t>((g.D + s_excl) & 15u) + my_excl;
+        sign = ld_u32_unaligned(pbuf, p) | (static_cast<uint64_t>(ld_u32_unaligned(pbuf, p + 4)) << 32);
+        p += 8;
+        if (is_o) {
+            outl = ld_u32_unaligned(pbuf, p);
+            if (nob < 4) outl &= (1u << (8 * nob)) - 1u;
+            p += nob;
+        }
+#pragma unroll
+        for (int k = 0; k < 32; k++) {
+            if (k < (int)fl) {
+                lo[k] = ld_u32_unaligned(pbuf, p + 8 * k);
+                hi[k] = ld_u32_unaligned(pbuf, p + 8 * k + 4);
+            }
+        }
+    }
+    if (flw > 0) {
+        if (flw <= 4) {
+            unpack_planes<2>(lo);
+            unpack_planes<2>(hi);
+        } else if (flw <= 8) {
+            unpack_planes<3>(lo);
+            unpack_planes<3>(hi);
+        } else if (flw <= 16) {
+            unpack_planes<4>(lo);
+            unpack_planes<4>(hi);
+        } else {
+            unpack_planes<5>(lo);
+            unpack_planes<5>(hi);
+        }
+    }
+    if (is_o) lo[0] = outl;
+    // ---- inverse nD Lorenzo in index order, ❶⁻¹, scatter to the field
+    int q[LND];
+#pragma unroll
+    for (int i = 0; i < LND; i++) {
+        const uint32_t m = i < 32 ? lo[i] : hi[i - 32];
+        const int d = ((sign >> i) & 1ull) ? -static_cast<int>(m) : static_cast<int>(m);
+        q[i] = d + lorenzo_pred<NDIM>(q, i);
+    }
+    if (active) {
+        const BlockOrigin bo = block_origin<NDIM>(g, b);
+#pragma unroll
+        for (int i = 0; i < LND; i++) {
+            const uint64_t idx = nd_index<NDIM>(g, bo, i);
+            if (idx != ~uint64_t(0)) out[idx] = dequantize(q[i], K.s);
+        }
+    }
+}
+
+}  // namespace cszp2

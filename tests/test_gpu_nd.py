@@ -1,0 +1,141 @@
+"""GPU parity for the multi-dimensional Lorenzo layouts (
+P:365-388, Table VI; FORMAT.md §7): 2D 8x8 and 3D 4x4x4 blocks through
+cszp2_compress_nd / cszp2_decompress_nd against oracle.compress_nd /
+oracle.decompress_nd — whole stream byte-identical (output pre-poisoned with
+0xAA), reconstruction bit-identical."""
+import numpy as np
+import pytest
+import torch
+
+pytestmark = pytest.mark.gpu
+
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+import oracle  # noqa: E402
+import paper_conf_sc_huangdlc24_b200 as cz  # noqa: E402
+
+DEV = torch.device("cuda:0")
+ENC = {"plain": oracle.PLAIN, "outlier": oracle.OUTLIER}
+EBM = {"abs": oracle.ABS, "rel": oracle.REL}
+
+
+def smooth_field(shape, seed, dtype, noise=1e-3):
+    """Seeded smooth field + small noise (the structure of the paper's 2D/3D
+    datasets: correlated along every axis)."""
+    rng = np.random.default_rng(seed)
+    axes = np.meshgrid(*[np.linspace(0, 3, s) for s in shape], indexing="ij")
+    f = np.ones(shape)
+    for k, a in enumerate(axes):
+        f = f * np.sin(a * (1.3 + 0.4 * k) + k) + 0.3 * np.cos(2.1 * a)
+    f = f + noise * rng.standard_normal(shape)
+    return f.astype(dtype)
+
+
+def gpu_nd(xh, eb, eb_mode, enc):
+    x = torch.from_numpy(xh).to(DEV)
+    out = torch.full((cz.compress_bound_nd(xh.shape, x.dtype),), 0xAA, dtype=torch.uint8, device=DEV)
+    nb = torch.zeros(1, dtype=torch.int64, device=DEV)
+    cz.compress_nd(x, eb, eb_mode, enc, out=out, out_bytes=nb)
+    torch.cuda.synchronize()
+    return x, out, int(nb.item())
+
+
+def check_nd(xh, eb, eb_mode, enc):
+    x, out, total = gpu_nd(xh, eb, eb_mode, enc)
+    ref, rc = oracle.compress_nd(xh, eb, EBM[eb_mode], ENC[enc])
+    got = out[:total].cpu().numpy()
+    assert total == ref.size
+    st = torch.zeros(1, dtype=torch.int32, device=DEV)
+    if rc == oracle.ERR_RANGE:
+        np.testing.assert_array_equal(got[:64], ref[:64])
+        cz.decompress_nd(out, xh.shape, x.dtype, status=st)
+        torch.cuda.synchronize()
+        assert int(st.item()) == 3
+        return got
+    assert rc == oracle.OK
+    if not np.array_equal(got, ref):
+        bad = np.nonzero(got != ref)[0]
+        raise AssertionError(f"stream differs at {bad.size} bytes, first {bad[:8]} (total {total})")
+    y = torch.full_like(x, float("nan"))
+    cz.decompress_nd(out, xh.shape, x.dtype, out=y, status=st)
+    torch.cuda.synchronize()
+    assert int(st.item()) == 0
+    yr, rc = oracle.decompress_nd(ref, xh.shape, xh.dtype)
+    assert rc == oracle.OK
+    iv = np.uint32 if xh.dtype == np.float32 else np.uint64
+    np.testing.assert_array_equal(y.cpu().numpy().view(iv), yr.view(iv))
+    return got
+
+
+SHAPES = [(8, 8), (37, 53), (1, 200), (300, 301), (0, 5),
+          (4, 4, 4), (9, 10, 11), (5, 17, 3), (33, 70, 65), (1, 1, 1)]
+
+
+@pytest.mark.parametrize("shape", SHAPES)
+@pytest.mark.parametrize("enc", ["plain", "outlier"])
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_nd_parity_rel(shape, enc, dtype):
+    xh = smooth_field(shape, sum(shape) + 3, dtype)
+    check_nd(xh, 1e-4, "rel", enc)
+
+
+@pytest.mark.parametrize("shape", [(300, 301), (33, 70, 65)])
+@pytest.mark.parametrize("eb", [0.5, 1e-2, 1e-6])
+def test_nd_parity_abs_noise(shape, eb):
+    rng = np.random.default_rng(7)
+    xh = rng.standard_normal(shape).astype(np.float32)
+    check_nd(xh, eb, "abs", "outlier")
+
+
+@pytest.mark.parametrize("ndim", [2, 3])
+def test_nd_range_status(ndim):
+    shape = (40, 40) if ndim == 2 else (12, 12, 12)
+    xh = smooth_field(shape, 1, np.float32)
+    xh.flat[777] = 1e30  # |x/2eb| beyond the predictor's limit
+    got = check_nd(xh, 1e-3, "abs", "outlier")
+    assert got[9] == 3
+
+
+def test_nd_and_1d_streams_are_not_interchangeable():
+    xh = smooth_field((64, 64), 5, np.float32)
+    x, out, total = gpu_nd(xh, 1e-3, "abs", "outlier")
+    st = torch.zeros(1, dtype=torch.int32, device=DEV)
+    cz.decompress(out, xh.size, torch.float32, status=st)
+    torch.cuda.synchronize()
+    assert int(st.item()) == 4
+    s1, _ = cz.compress(x.view(-1), 1e-3, "abs", "outlier")
+    st.zero_()
+    cz.decompress_nd(s1, xh.shape, torch.float32, status=st)
+    torch.cuda.synchronize()
+    assert int(st.item()) == 4
+    st.zero_()  # wrong extents
+    cz.decompress_nd(out, (32, 128), torch.float32, status=st)
+    torch.cuda.synchronize()
+    assert int(st.item()) == 4
+
+
+def test_nd_bad_arguments():
+    x = torch.zeros(4, 4, 4, device=DEV)
+    out = torch.empty(cz.compress_bound_nd((4, 4, 4)), dtype=torch.uint8, device=DEV)
+    rc = cz._lib.cszp2_compress_nd(cz._ptr(x), 4, 4, 4, 2, 0, 1e-3, 0, 1, cz._ptr(out), None,
+                                   cz._stream(None))  # ndim 2 with nz != 1
+    assert rc == cz.ERR_ARG
+    assert cz._lib.cszp2_compress_bound_nd(4, 4, 4, 4, 0) == 0
+    assert cz._lib.cszp2_compress_bound_nd(1 << 32, 1, 1, 2, 0) == 0
+
+
+@pytest.mark.parametrize("ndim", [2, 3])
+def test_nd_error_bound_and_ratio_vs_1d(ndim):
+    """Table VI analog: on a smooth field the nD predictor beats the 1D one
+    in compression ratio; both honour the bound."""
+    shape = (512, 512) if ndim == 2 else (64, 64, 64)
+    xh = smooth_field(shape, 11, np.float32, noise=0.0)
+    x, out, total = gpu_nd(xh, 1e-4, "rel", "outlier")
+    y = cz.decompress_nd(out, xh.shape, torch.float32)
+    s1, n1 = cz.compress(x.view(-1), 1e-4, "rel", "outlier")
+    torch.cuda.synchronize()
+    eb_abs = float(np.frombuffer(out[32:40].cpu().numpy().tobytes(), dtype=np.float64)[0])
+    err = (y.double() - x.double()).abs().max().item()
+    assert err <= eb_abs * (1 + 1e-6) + 1e-7 * float(x.abs().max())
+    assert total < int(n1.item())
