@@ -162,7 +162,7 @@ int cszp2_container_index(const uint64_t *d_sizes, int nparts, uint64_t *d_offse
  * cszp2_compress_nd: like cszp2_compress (same eb / eb_mode / enc_mode meaning,
  *   same RANGE behaviour with this predictor's tighter limit |x/2eb| <= 2^28-1 (2D)
  *   or 2^27-1 (3D), FORMAT.md §7); asynchronous on `stream`.
- * cszp2_decompress_nd: inverse; d_out = nx*ny*nz values (any 4/8-byte alignment);
+ * cszp2_decompress_nd: inverse; d_out = nx*ny*nz values, device, 16-byte aligned;
  *   d_status as in cszp2_decompress. */
 uint64_t cszp2_compress_bound_nd(uint64_t nx, uint64_t ny, uint64_t nz, int ndim, int dtype);
 int cszp2_compress_nd(const void *d_in, uint64_t nx, uint64_t ny, uint64_t nz, int ndim, int dtype,

@@ -431,7 +431,7 @@ int cszp2_decompress_nd(const void *d_cmp, void *d_out, uint64_t nx, uint64_t ny
                         int dtype, int *d_status, void *stream) {
     GeomND g;
     if (!wsize(dtype) || !d_cmp || geometry_nd(nx, ny, nz, ndim, &g)) return CSZP2_ERR_ARG;
-    if ((!d_out && g.n) || !aligned16(d_cmp)) return CSZP2_ERR_ARG;
+    if ((!d_out && g.n) || !aligned16(d_cmp) || (g.n && !aligned16(d_out))) return CSZP2_ERR_ARG;
     cudaStream_t st = S(stream);
     if (dtype == CSZP2_F32)
         return ndim == 2 ? launch_decompress_nd<float, 2>(d_cmp, d_out, g, d_status, st)

@@ -82,6 +82,29 @@ __device__ __forceinline__ uint64_t nd_index(const GeomND &g, const BlockOrigin 
     return (z * g.ny + y) * g.nx + x;
 }
 
+// 16-byte vectors of the value type (rows of a block are 4 or 8 contiguous values)
+template <typename T>
+struct Vec16;
+template <>
+struct Vec16<float> {
+    using type = float4;
+    static constexpr int V = 4;
+};
+template <>
+struct Vec16<double> {
+    using type = double2;
+    static constexpr int V = 2;
+};
+
+// true if block b lies entirely inside the field and its rows are 16-byte aligned
+// (x extent a multiple of the vector width; the base is 16-byte aligned by the ABI)
+template <typename T, int NDIM>
+__device__ __forceinline__ bool interior_vec(const GeomND &g, const BlockOrigin &o) {
+    using S = BlockShape<NDIM>;
+    return (g.nx % Vec16<T>::V) == 0 && o.x0 + S::BX <= g.nx && o.y0 + S::BY <= g.ny &&
+           o.z0 + S::BZ <= g.nz;
+}
+
 // one 32-bit word to smem at any byte position (neighbouring blocks own the other bytes)
 __device__ __forceinline__ void put_word(uint8_t *base, uint32_t pos, uint32_t w) {
     if ((pos & 3u) == 0) {
@@ -124,14 +147,34 @@ __global__ void __launch_bounds__(NT) compress_nd_kernel(const T *__restrict__ i
     uint64_t outside = 0;  // bit i: value i lies outside the field
     bool bad = false;
     const BlockOrigin bo = block_origin<NDIM>(g, active ? b : 0);
+    if (active && interior_vec<T, NDIM>(g, bo)) {
+        // interior block: each row of BX values by 16-byte loads
+        using S = BlockShape<NDIM>;
+        using VT = typename Vec16<T>::type;
+        constexpr int V = Vec16<T>::V;
 #pragma unroll
-    for (int i = 0; i < LND; i++) {
-        const uint64_t idx = active ? nd_index<NDIM>(g, bo, i) : ~uint64_t(0);
-        q[i] = 0;
-        if (idx != ~uint64_t(0))
-            q[i] = quantize_nd<NDIM>(in[idx], K.inv, bad);
-        else
-            outside |= 1ull << i;
+        for (int r = 0; r < S::BY * S::BZ; r++) {
+            const int iy = r % S::BY, iz = r / S::BY;
+            const VT *row = reinterpret_cast<const VT *>(
+                in + ((bo.z0 + iz) * g.ny + bo.y0 + iy) * g.nx + bo.x0);
+#pragma unroll
+            for (int v = 0; v < S::BX / V; v++) {
+                T tmp[V];
+                *reinterpret_cast<VT *>(tmp) = __ldg(row + v);
+#pragma unroll
+                for (int k = 0; k < V; k++) q[r * S::BX + v * V + k] = quantize_nd<NDIM>(tmp[k], K.inv, bad);
+            }
+        }
+    } else {
+#pragma unroll
+        for (int i = 0; i < LND; i++) {
+            const uint64_t idx = active ? nd_index<NDIM>(g, bo, i) : ~uint64_t(0);
+            q[i] = 0;
+            if (idx != ~uint64_t(0))
+                q[i] = quantize_nd<NDIM>(in[idx], K.inv, bad);
+            else
+                outside |= 1ull << i;
+        }
     }
     // ---- nD Lorenzo residuals, highest index first so every prediction still sees q
     uint32_t a[LND];
@@ -386,10 +429,28 @@ __global__ void __launch_bounds__(NT) decompress_nd_kernel(const uint8_t *__rest
     }
     if (active) {
         const BlockOrigin bo = block_origin<NDIM>(g, b);
+        if (interior_vec<T, NDIM>(g, bo)) {
+            using S = BlockShape<NDIM>;
+            using VT = typename Vec16<T>::type;
+            constexpr int V = Vec16<T>::V;
 #pragma unroll
-        for (int i = 0; i < LND; i++) {
-            const uint64_t idx = nd_index<NDIM>(g, bo, i);
-            if (idx != ~uint64_t(0)) out[idx] = dequantize(q[i], K.s);
+            for (int r = 0; r < S::BY * S::BZ; r++) {
+                const int iy = r % S::BY, iz = r / S::BY;
+                VT *row = reinterpret_cast<VT *>(out + ((bo.z0 + iz) * g.ny + bo.y0 + iy) * g.nx + bo.x0);
+#pragma unroll
+                for (int v = 0; v < S::BX / V; v++) {
+                    T tmp[V];
+#pragma unroll
+                    for (int k = 0; k < V; k++) tmp[k] = dequantize(q[r * S::BX + v * V + k], K.s);
+                    row[v] = *reinterpret_cast<VT *>(tmp);
+                }
+            }
+        } else {
+#pragma unroll
+            for (int i = 0; i < LND; i++) {
+                const uint64_t idx = nd_index<NDIM>(g, bo, i);
+                if (idx != ~uint64_t(0)) out[idx] = dequantize(q[i], K.s);
+            }
         }
     }
 }
