@@ -1,0 +1,83 @@
+"""Compression-accelerated all-gather (the paper's motivating
+use, P:67-77 — "compressing data before [GPU-to-GPU] transfer … reduces the volume
+of data", gZCCL-style collectives P:491-495).
+
+Every rank holds an equal-sized shard x_r (n values). Instead of moving n·w bytes
+per rank, each rank
+
+  1. compresses its shard with the single-kernel compressor (cszp2_compress),
+  2. all-gathers the 8-byte compressed sizes (NCCL, device to device),
+  3. all-gathers the compressed streams in slots of the largest size (one NCCL
+     all_gather_into_tensor; one 8-byte device->host read to size the slots),
+  4. decompresses every rank's stream into its slice of the output.
+
+The result equals all_gather(decompress(compress(x_r))) bit for bit; the bytes on
+the wire are world · max_r(stream_r) instead of world · n·w. Error bound: each
+shard's own (per-rank REL uses the shard's range, R-21).
+
+The codec is the CUDA one; `codec=` exists so the host-side logic can be tested
+with world-size-2 gloo on CPU (tests/test_multi_gloo.py passes a test-only codec).
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import torch
+import torch.distributed as dist
+
+from .multi import gather_sizes
+
+
+@dataclass
+class CudaCodec:
+    """The product codec: libcszp2 kernels on CUDA tensors."""
+
+    eb: float
+    eb_mode: str = "rel"
+    enc_mode: str = "outlier"
+
+    def compress(self, x: torch.Tensor, stream=None):
+        from . import compress
+
+        return compress(x, self.eb, self.eb_mode, self.enc_mode, stream=stream)
+
+    def decompress(self, cmp: torch.Tensor, n: int, out: torch.Tensor, stream=None):
+        from . import decompress
+
+        decompress(cmp, n, out.dtype, out=out, stream=stream)
+
+
+def _all_gather_bytes(recv: torch.Tensor, send: torch.Tensor, group=None):
+    if send.is_cuda:
+        dist.all_gather_into_tensor(recv, send, group=group)
+    else:  # gloo (host-logic tests)
+        parts = list(recv.split(send.numel()))
+        dist.all_gather(parts, send, group=group)
+        recv.copy_(torch.cat(parts))
+
+
+def compressed_all_gather(x: torch.Tensor, eb: float, eb_mode: str = "rel", enc_mode: str = "outlier",
+                          group=None, codec=None, out: torch.Tensor | None = None, stats: dict | None = None):
+    """All-gather equal-sized shards through the compressor. Returns a tensor of
+    world·n values (rank order), like all_gather_into_tensor of the lossy shards.
+    `stats` (optional dict) receives the per-rank stream sizes and wire bytes."""
+    codec = codec or CudaCodec(eb, eb_mode, enc_mode)
+    x = x.contiguous().view(-1)
+    world = dist.get_world_size(group)
+    n, w = x.numel(), x.element_size()
+    if (n * w) % 16:
+        raise ValueError("shard size must be a multiple of 16 bytes (output slices stay 16-byte aligned)")
+    if out is None:
+        out = torch.empty(world * n, dtype=x.dtype, device=x.device)
+    buf, nbytes = codec.compress(x)                 # 1. one fused compression kernel
+    sizes = gather_sizes(nbytes.view(1), group)     # 2. 8 B per rank over NCCL
+    slot = (int(sizes.max().item()) + 15) // 16 * 16  # the one host read
+    if slot > buf.numel():
+        raise RuntimeError("compressed stream larger than its buffer")
+    recv = torch.empty(world * slot, dtype=torch.uint8, device=x.device)
+    _all_gather_bytes(recv, buf[:slot], group)      # 3. the compressed payloads
+    for r in range(world):                          # 4. P decompression kernels
+        codec.decompress(recv[r * slot:(r + 1) * slot], n, out[r * n:(r + 1) * n])
+    if stats is not None:
+        stats.update(sizes=sizes.tolist(), slot=slot, wire_bytes=world * slot, raw_bytes=world * n * w)
+    return out

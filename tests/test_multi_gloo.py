@@ -91,3 +91,75 @@ def test_slab_edge_cases():
                 assert a + c == b
                 assert b % 32 == 0 or b == n
     assert slab(2**33, 8, 3) == (3 * 2**30, 2**30)
+
+
+class _OracleCodec:
+    """Test-only codec for the host logic of the compressed all-gather on CPU: the
+    oracle behind the same (compress, decompress) interface as CudaCodec."""
+
+    def __init__(self, eb, eb_mode, enc):
+        self.eb, self.eb_mode, self.enc = eb, eb_mode, enc
+
+    def compress(self, x):
+        import oracle
+
+        s, rc = oracle.compress(x.numpy(), self.eb, self.eb_mode, self.enc)
+        assert rc == oracle.OK
+        buf = torch.zeros(oracle.compress_bound(x.numel()) + 16, dtype=torch.uint8)
+        buf[: s.size] = torch.from_numpy(s)
+        return buf, torch.tensor([s.size], dtype=torch.int64)
+
+    def decompress(self, cmp, n, out):
+        import oracle
+
+        y, rc = oracle.decompress(cmp.numpy(), n, np.float32 if out.dtype == torch.float32 else np.float64)
+        assert rc == oracle.OK
+        out.copy_(torch.from_numpy(y))
+
+
+def _cag_worker(rank, world, port, n, eb, enc, result_q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_sc_huangdlc24_b200.collective import compressed_all_gather
+        from synthetic import make_field
+
+        x = make_field("cfg2", "cpu", rank * n, n)  # shard r of one field
+        stats = {}
+        y = compressed_all_gather(x, eb, "rel", "outlier", codec=_OracleCodec(eb, 1, enc), stats=stats)
+        result_q.put((rank, y.numpy().tobytes(), stats))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("enc", [0, 1])
+def test_compressed_all_gather_two_ranks(orc, enc):
+    """NEXT #4 host logic: sizes all-gathered, payloads gathered in max-size slots,
+    every rank ends with the same world·n values = each shard's lossy round trip."""
+    world, n, eb = 2, 3 * 8192 + 32 * 7 + 4, 1e-4
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_cag_worker, args=(r, world, port, n, eb, enc, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted([q.get(timeout=120) for _ in range(world)], key=lambda r: r[0])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    from synthetic import make_field
+
+    expect, sizes = [], []
+    for r in range(world):
+        x = make_field("cfg2", "cpu", r * n, n).numpy()
+        s, rc = orc.compress(x, eb, orc.REL, enc)
+        sizes.append(s.size)
+        y, rc = orc.decompress(s, n, np.float32)
+        expect.append(y)
+    expect = np.concatenate(expect)
+    for rank, yb, stats in res:
+        np.testing.assert_array_equal(np.frombuffer(yb, np.float32).view(np.uint32), expect.view(np.uint32))
+        assert stats["sizes"] == sizes
+        assert stats["slot"] == (max(sizes) + 15) // 16 * 16
+        assert stats["wire_bytes"] == world * stats["slot"] < stats["raw_bytes"]
