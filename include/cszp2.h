@@ -90,10 +90,18 @@ int cszp2_compress_prepare(const void *d_in, uint64_t n, int dtype, double eb, i
 int cszp2_compress_encode(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
                           int enc_mode, void *d_out, uint64_t *d_out_bytes, void *stream);
 
-/* cszp2_compress_encode with ablation flags (same stream bytes either way):
+/* cszp2_compress_encode with ablation flags (NEXT #2; same stream bytes either way):
  *  CSZP2_FLAG_CHAINED_SCAN: replace the decoupled lookback by the plain chained
- *  scan it improves on (Fig 12 left; the Fig 17 comparison). */
+ *    scan it improves on (Fig 12 left; the Fig 17 comparison).
+ *  CSZP2_FLAG_LOAD_VEC: each thread loads its own 32-value block with 16-byte
+ *    vector loads (the paper's vectorised access, Fig 10-11) instead
+ *    of the TMA tensor tiles.
+ *  CSZP2_FLAG_LOAD_SCALAR: each thread loads its block value by value (the
+ *    non-vectorised baseline of the §VI-E memory ablation).
+ *  LOAD_VEC and LOAD_SCALAR are exclusive (ARG otherwise). */
 #define CSZP2_FLAG_CHAINED_SCAN 1u
+#define CSZP2_FLAG_LOAD_VEC 2u
+#define CSZP2_FLAG_LOAD_SCALAR 4u
 int cszp2_compress_encode_ex(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
                              int enc_mode, void *d_out, uint64_t *d_out_bytes, unsigned flags,
                              void *stream);
@@ -108,6 +116,22 @@ int cszp2_compress_encode_ex(const void *d_in, uint64_t n, int dtype, double eb,
  *             caller zeroes it beforehand. */
 int cszp2_decompress(const void *d_cmp, void *d_out, uint64_t n, int dtype, int *d_status,
                      void *stream);
+
+/* Ablation (NEXT #2): a one-CTA-per-tile decompression kernel in two variants
+ * that differ only in how a tile's payload start is found:
+ *  CSZP2_LOCATE_LOOKBACK: the paper's way (❸ runs again in decompression)
+ *    — the tile's payload bytes recomputed from its offset bytes, then a
+ *    decoupled lookback over a caller-provided scratch array;
+ *  CSZP2_LOCATE_INDEX: read from the persisted tile index (R-14).
+ * Same output as cszp2_decompress.
+ *  d_scratch : cszp2_decompress_scratch_bytes(n) bytes of device memory, zeroed
+ *              by this call (asynchronously, on `stream`; used by LOOKBACK).
+ *  other arguments as cszp2_decompress; ARG for an unknown `locate`. */
+#define CSZP2_LOCATE_INDEX 0
+#define CSZP2_LOCATE_LOOKBACK 1
+uint64_t cszp2_decompress_scratch_bytes(uint64_t n);
+int cszp2_decompress_tilewise(const void *d_cmp, void *d_out, uint64_t n, int dtype, int locate,
+                              void *d_scratch, int *d_status, void *stream);
 
 /* Random-access decompression (§VI-B): decode only the values
  * [first, first + count) of a stream of n values into d_out[0 .. count)

@@ -68,6 +68,9 @@ def _load():
                                       ctypes.POINTER(ctypes.c_uint64), vp]
     L.cszp2_decompress_host.argtypes = [vp, u64, vp, vp, vp, u64, i32, vp, vp]
     L.cszp2_container_index.argtypes = [vp, i32, vp, vp]
+    L.cszp2_decompress_scratch_bytes.argtypes = [u64]
+    L.cszp2_decompress_scratch_bytes.restype = u64
+    L.cszp2_decompress_tilewise.argtypes = [vp, vp, u64, i32, i32, vp, vp, vp]
     L.cszp2_compress_bound_nd.argtypes = [u64, u64, u64, i32, i32]
     L.cszp2_compress_bound_nd.restype = u64
     L.cszp2_compress_nd.argtypes = [vp, u64, u64, u64, i32, i32, dbl, i32, i32, vp, vp, vp]
@@ -84,6 +87,7 @@ EXPORTED = (
     "cszp2_decompress", "cszp2_decompress_range", "cszp2_read_header", "cszp2_compress_host", "cszp2_decompress_host",
     "cszp2_container_index", "cszp2_version",
     "cszp2_compress_bound_nd", "cszp2_compress_nd", "cszp2_decompress_nd",
+    "cszp2_decompress_scratch_bytes", "cszp2_decompress_tilewise",
 )
 
 
@@ -149,10 +153,13 @@ def compress_encode(x, eb, eb_mode, enc_mode, out, out_bytes=None, stream=None):
 
 
 FLAG_CHAINED_SCAN = 1
+FLAG_LOAD_VEC = 2
+FLAG_LOAD_SCALAR = 4
 
 
 def compress_encode_ex(x, eb, eb_mode, enc_mode, out, out_bytes=None, flags=0, stream=None):
-    """compress_encode with ablation flags (FLAG_CHAINED_SCAN: plain chained scan)."""
+    """compress_encode with ablation flags (FLAG_CHAINED_SCAN: plain chained scan;
+    FLAG_LOAD_VEC / FLAG_LOAD_SCALAR: per-thread global loads instead of TMA)."""
     rc = _lib.cszp2_compress_encode_ex(_ptr(x), x.numel(), _DT[x.dtype], float(eb), _EB[eb_mode],
                                        _ENC[enc_mode], _ptr(out), _ptr(out_bytes), flags, _stream(stream))
     _check("cszp2_compress_encode_ex", rc)
@@ -166,6 +173,24 @@ def decompress(cmp: torch.Tensor, n: int, dtype=torch.float32, out=None, status=
         out = torch.empty(n, dtype=dtype, device=cmp.device)
     rc = _lib.cszp2_decompress(_ptr(cmp), _ptr(out), n, _DT[out.dtype], _ptr(status), _stream(stream))
     _check("cszp2_decompress", rc)
+    return out
+
+
+LOCATE_INDEX, LOCATE_LOOKBACK = 0, 1
+
+
+def decompress_tilewise(cmp: torch.Tensor, n: int, dtype=torch.float32, locate=LOCATE_LOOKBACK, out=None,
+                        scratch=None, status=None, stream=None):
+    """Ablation: one-CTA-per-tile decompression locating tiles by a decoupled lookback
+    (the paper's decompression-side ❸) or by the persisted tile index."""
+    _need_cuda(cmp, out, scratch, status)
+    if out is None:
+        out = torch.empty(n, dtype=dtype, device=cmp.device)
+    if scratch is None:
+        scratch = torch.empty(int(_lib.cszp2_decompress_scratch_bytes(n)), dtype=torch.uint8, device=cmp.device)
+    rc = _lib.cszp2_decompress_tilewise(_ptr(cmp), _ptr(out), n, _DT[out.dtype], int(locate), _ptr(scratch),
+                                        _ptr(status), _stream(stream))
+    _check("cszp2_decompress_tilewise", rc)
     return out
 
 

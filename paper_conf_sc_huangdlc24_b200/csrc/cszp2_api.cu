@@ -126,16 +126,17 @@ int launch_minmax(const void *d_in, uint64_t n, double lambda, void *d_out, cuda
     return launch_status();
 }
 
-template <typename T, bool OUTLIER>
-int launch_compress(const void *d_in, const Geom &g, double eb, int eb_mode, int enc_mode,
-                    void *d_out, uint64_t *d_out_bytes, cudaStream_t st, unsigned flags) {
+template <typename T, bool OUTLIER, int LOAD>
+int launch_compress_l(const void *d_in, const Geom &g, double eb, int eb_mode, int enc_mode,
+                      void *d_out, uint64_t *d_out_bytes, cudaStream_t st, unsigned flags) {
     static std::once_flag once;
     static int attr_rc = CSZP2_OK;
     static int grid_cache = 0;
     constexpr int smem = compress_smem_bytes<T>();
-    std::call_once(once, [] { attr_rc = set_smem(compress_kernel<T, OUTLIER>, smem); });
+    std::call_once(once, [] { attr_rc = set_smem(compress_kernel<T, OUTLIER, LOAD>, smem); });
     if (attr_rc) return attr_rc;
-    const unsigned grid = persistent_grid(compress_kernel<T, OUTLIER>, NT_COMP, smem, g.T, &grid_cache);
+    const unsigned grid =
+        persistent_grid(compress_kernel<T, OUTLIER, LOAD>, NT_COMP, smem, g.T, &grid_cache);
     unsigned *ticket = reinterpret_cast<unsigned *>(static_cast<uint8_t *>(d_out) + stream_bound(g));
     CUtensorMap map;
     int rc = make_tmap(&map, d_in, Traits<T>::DTYPE, g.nfull);
@@ -146,10 +147,20 @@ int launch_compress(const void *d_in, const Geom &g, double eb, int eb_mode, int
     hs.eb_mode = static_cast<uint32_t>(eb_mode);
     hs.eb_user = eb;
     hs.flags = flags;
-    compress_kernel<T, OUTLIER><<<grid, NT_COMP, smem, st>>>(
+    compress_kernel<T, OUTLIER, LOAD><<<grid, NT_COMP, smem, st>>>(
         map, static_cast<const T *>(d_in), g, eb, eb_mode == CSZP2_EB_REL ? 1 : 0,
         static_cast<uint8_t *>(d_out), ticket, d_out_bytes, hs);
     return launch_status();
+}
+
+template <typename T, bool OUTLIER>
+int launch_compress(const void *d_in, const Geom &g, double eb, int eb_mode, int enc_mode,
+                    void *d_out, uint64_t *d_out_bytes, cudaStream_t st, unsigned flags) {
+    if (flags & CSZP2_FLAG_LOAD_VEC)
+        return launch_compress_l<T, OUTLIER, LOAD_VEC>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags);
+    if (flags & CSZP2_FLAG_LOAD_SCALAR)
+        return launch_compress_l<T, OUTLIER, LOAD_SCALAR>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags);
+    return launch_compress_l<T, OUTLIER, LOAD_TMA>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags);
 }
 
 template <typename T>
@@ -283,7 +294,8 @@ int cszp2_compress_encode_ex(const void *d_in, uint64_t n, int dtype, double eb,
     int rc = check_compress_args(d_in, n, dtype, eb, eb_mode, d_out);
     if (rc) return rc;
     if (enc_mode != CSZP2_ENC_PLAIN && enc_mode != CSZP2_ENC_OUTLIER) return CSZP2_ERR_ARG;
-    if (flags & ~1u) return CSZP2_ERR_ARG;
+    if (flags & ~(CSZP2_FLAG_CHAINED_SCAN | CSZP2_FLAG_LOAD_VEC | CSZP2_FLAG_LOAD_SCALAR)) return CSZP2_ERR_ARG;
+    if ((flags & CSZP2_FLAG_LOAD_VEC) && (flags & CSZP2_FLAG_LOAD_SCALAR)) return CSZP2_ERR_ARG;
     Geom g = geometry(n);
     cudaStream_t st = S(stream);
     if (dtype == CSZP2_F32)
@@ -317,6 +329,40 @@ int cszp2_decompress(const void *d_cmp, void *d_out, uint64_t n, int dtype, int 
     Geom g = geometry(n);
     return dtype == CSZP2_F32 ? launch_decompress<float>(d_cmp, d_out, g, d_status, S(stream))
                               : launch_decompress<double>(d_cmp, d_out, g, d_status, S(stream));
+}
+
+uint64_t cszp2_decompress_scratch_bytes(uint64_t n) {
+    const Geom g = geometry(n);
+    return 8 * (g.T ? g.T : 1) + 16;  // descriptors + ticket
+}
+
+int cszp2_decompress_tilewise(const void *d_cmp, void *d_out, uint64_t n, int dtype, int locate,
+                              void *d_scratch, int *d_status, void *stream) {
+    if (!wsize(dtype) || !d_cmp || !d_scratch || (!d_out && n)) return CSZP2_ERR_ARG;
+    if (locate != CSZP2_LOCATE_INDEX && locate != CSZP2_LOCATE_LOOKBACK) return CSZP2_ERR_ARG;
+    if (!aligned16(d_cmp) || (n && !aligned16(d_out)) || n > (1ull << 40)) return CSZP2_ERR_ARG;
+    const Geom g = geometry(n);
+    cudaStream_t st = S(stream);
+    if (cudaMemsetAsync(d_scratch, 0, cszp2_decompress_scratch_bytes(n), st) != cudaSuccess)
+        return CSZP2_ERR_CUDA;
+    const unsigned grid = static_cast<unsigned>(g.T ? g.T : 1);
+    uint64_t *scr = static_cast<uint64_t *>(d_scratch);
+    const uint8_t *c = static_cast<const uint8_t *>(d_cmp);
+    const bool lb = locate == CSZP2_LOCATE_LOOKBACK;
+    if (dtype == CSZP2_F32) {
+        float *o = static_cast<float *>(d_out);
+        if (lb)
+            decompress_tilewise_kernel<float, true><<<grid, NT, 0, st>>>(c, o, g, scr, d_status);
+        else
+            decompress_tilewise_kernel<float, false><<<grid, NT, 0, st>>>(c, o, g, scr, d_status);
+    } else {
+        double *o = static_cast<double *>(d_out);
+        if (lb)
+            decompress_tilewise_kernel<double, true><<<grid, NT, 0, st>>>(c, o, g, scr, d_status);
+        else
+            decompress_tilewise_kernel<double, false><<<grid, NT, 0, st>>>(c, o, g, scr, d_status);
+    }
+    return launch_status();
 }
 
 int cszp2_decompress_range(const void *d_cmp, uint64_t n, int dtype, uint64_t first,

@@ -664,7 +664,12 @@ __device__ __forceinline__ void write_payload(const uint8_t *stg, uint8_t *out, 
     }
 }
 
-template <typename T, bool OUTLIER>
+// LOAD (NEXT #2 memory ablation, Fig 10-11): 0 = TMA tensor tiles (the
+// product path), 1 = each thread reads its own block with 16-byte vector loads (the
+// paper's vectorised access), 2 = each thread reads its block value by value.
+constexpr int LOAD_TMA = 0, LOAD_VEC = 1, LOAD_SCALAR = 2;
+
+template <typename T, bool OUTLIER, int LOAD = LOAD_TMA>
 __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kernel(
     const __grid_constant__ CUtensorMap tmap, const T *__restrict__ in, const Geom g,
     const double eb_abs_arg, const int eb_from_header, uint8_t *__restrict__ out,
@@ -695,7 +700,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
     // s_full so its phase advances even without data)
     auto issue = [&](uint64_t tk) {
         const uint64_t b0 = tk * BPT;
-        if (b0 < g.nfull) {
+        if (LOAD == LOAD_TMA && b0 < g.nfull) {
             if (Traits<T>::ROWS == 1) {
                 mbar_expect_tx(&s_full, BPT * 128);
                 tma_load_2d(inbuf, &tmap, 0, static_cast<int>(b0), &s_full);
@@ -756,8 +761,16 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
 
             T x[L];
             uint32_t valid = L;
-            if (full) {
+            if (full && LOAD == LOAD_TMA) {
                 load_block(inbuf, tid, x);
+            } else if (full && LOAD == LOAD_VEC) {
+                const uint4 *src = reinterpret_cast<const uint4 *>(in + b * L);
+#pragma unroll
+                for (int v = 0; v < L * (int)sizeof(T) / 16; v++)
+                    *reinterpret_cast<uint4 *>(reinterpret_cast<uint8_t *>(x) + 16 * v) = __ldg(src + v);
+            } else if (full) {
+#pragma unroll
+                for (int i = 0; i < L; i++) x[i] = __ldg(in + b * L + i);
             } else {
                 valid = active ? static_cast<uint32_t>(g.n - b * L) : 0u;
 #pragma unroll
@@ -1311,6 +1324,92 @@ __global__ void __launch_bounds__(NT) decompress_range_kernel(const uint8_t *__r
     for (int i = 0; i < L; i++) {
         const uint64_t v = v0 + i;
         if (v >= first && v < last && v < g.n) out[v - first] = x[i];
+    }
+}
+
+// Ablation (NEXT #2): one CTA per tile in ticket order. LOOKBACK = the paper's
+// decompression-side ❸: the tile's payload bytes are recomputed from its offset
+// bytes, then a decoupled lookback over the scratch descriptors gives the tile's payload
+// start. !LOOKBACK = the same kernel reading the start from the persisted tile index
+// (R-14), so the two differ only in how the tile is located.
+template <typename T, bool LOOKBACK>
+__global__ void __launch_bounds__(NT) decompress_tilewise_kernel(const uint8_t *__restrict__ cmp,
+                                                                 T *__restrict__ out, const Geom g,
+                                                                 uint64_t *__restrict__ scratch,
+                                                                 int *__restrict__ d_status) {
+    __shared__ __align__(16) uint8_t pbuf[PBUF_BYTES];
+    __shared__ uint64_t s_bar;
+    __shared__ uint32_t s_warp[NT / 32];
+    __shared__ uint64_t s_excl;
+    __shared__ double s_eb;
+    __shared__ int s_err;
+    __shared__ uint32_t s_tk;
+    const int tid = threadIdx.x;
+    unsigned *ticket = reinterpret_cast<unsigned *>(scratch + (g.T ? g.T : 1));
+    if (tid == 0) {
+        s_tk = atomicAdd(ticket, 1u);
+        double eb;
+        uint64_t pb;
+        s_err = check_header<T>(cmp, g, &eb, &pb);
+        s_eb = eb;
+        mbar_init(&s_bar, 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    const uint64_t t = s_tk;
+    // every CTA publishes (also on error) so no successor waits forever
+    const uint64_t b = t * BPT + tid;
+    const bool active = b < g.nb && !s_err;
+    const uint32_t obyte = active ? cmp[g.O + b] : 0u;
+    const uint32_t fl = obyte & 31u;
+    const bool is_o = (obyte & 0x80u) != 0;
+    const uint32_t nob = is_o ? ((obyte >> 5) & 3u) + 1u : 0u;
+    bool bad = (!is_o && (obyte & 0x60u));
+    const uint32_t size = is_o ? 4u + nob + 4u * fl : (fl ? 4u * (1u + fl) : 0u);
+    uint32_t agg;
+    const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg);
+    const bool any_bad = __syncthreads_or(bad);
+    if (tid < 32) {
+        uint64_t e = 0;
+        bool rng = false;
+        if (LOOKBACK) {
+            if (tid == 0) publish_aggregate(scratch, t, agg, false);
+            __syncwarp();
+            if (t > 0) e = lookback(scratch, t, agg, false, &rng);
+        } else if (t > 0 && t < g.T && !s_err) {
+            const uint64_t d = reinterpret_cast<const uint64_t *>(cmp)[8 + t - 1];
+            e = d & VAL_MASK;
+        }
+        if (tid == 0) {
+            s_excl = e;
+            if (!s_err && !any_bad && agg > 0) {
+                const uint64_t src0 = (g.D + e) & ~uint64_t(15);
+                const uint32_t len = static_cast<uint32_t>(roundup16(g.D + e + agg) - src0);
+                mbar_expect_tx(&s_bar, len);
+                bulk_load(pbuf, cmp + src0, len, &s_bar);
+            } else {
+                mbar_expect_tx(&s_bar, 0);
+            }
+        }
+    }
+    __syncthreads();
+    if (s_err || any_bad) {
+        if (tid == 0 && d_status) atomicOr(d_status, s_err ? s_err : ST_FORMAT);
+        return;
+    }
+    mbar_wait(&s_bar, 0);
+    const auto K = make_consts(s_eb, static_cast<T *>(nullptr));
+    T x[L];
+    decode_block(pbuf, static_cast<uint32_t>((g.D + s_excl) & 15u) + my_excl, obyte, size, K.s, x);
+    if (b < g.nfull) {
+        uint4 *dst = reinterpret_cast<uint4 *>(out + b * L);
+#pragma unroll
+        for (int v = 0; v < L * (int)sizeof(T) / 16; v++)
+            dst[v] = *reinterpret_cast<const uint4 *>(reinterpret_cast<const uint8_t *>(x) + 16 * v);
+    } else if (b < g.nb) {
+#pragma unroll
+        for (int i = 0; i < L; i++)
+            if (b * L + i < g.n) out[b * L + i] = x[i];
     }
 }
 

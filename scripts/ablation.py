@@ -1,5 +1,7 @@
 """NEXT rows measured on B200: (#2) decoupled lookback vs plain chained scan
-(the paper's Fig 17 comparison) and (#1) random-access decompression
+(the paper's Fig 17 comparison), TMA vs per-thread vector vs scalar
+loads (the §VI-E memory ablation), persisted tile index vs the paper's
+decompression-side lookback (R-14), and (#1) random-access decompression
 (P:345-356). Prints one JSON object; timings with CUDA events after warm-up."""
 import json, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -28,7 +30,8 @@ for cfg in sys.argv[1:] or ["cfg3b", "cfg5"]:
     lam = spec.ebs[-1]
     r = {}
     t_prep = timeit(lambda: cz.compress_prepare(x, lam, spec.eb_mode, out))
-    for name, flags in (("decoupled_lookback", 0), ("chained_scan", cz.FLAG_CHAINED_SCAN)):
+    for name, flags in (("decoupled_lookback", 0), ("chained_scan", cz.FLAG_CHAINED_SCAN),
+                        ("load_vec16_per_thread", cz.FLAG_LOAD_VEC), ("load_scalar_per_thread", cz.FLAG_LOAD_SCALAR)):
         def run():
             cz.compress_prepare(x, lam, spec.eb_mode, out)
             cz.compress_encode_ex(x, lam, spec.eb_mode, "outlier", out, nb, flags=flags)
@@ -38,6 +41,8 @@ for cfg in sys.argv[1:] or ["cfg3b", "cfg5"]:
         r[name] = {"compress_kernel_ms": round(t * 1e3, 4), "gbs_uncompressed": round(n * w / t / 1e9, 1),
                    "roofline_gbs": round((n * w + total) / t / 1e9, 1)}
     r["lookback_speedup"] = round(r["chained_scan"]["compress_kernel_ms"] / r["decoupled_lookback"]["compress_kernel_ms"], 2)
+    r["tma_vs_vec_speedup"] = round(r["load_vec16_per_thread"]["compress_kernel_ms"] / r["decoupled_lookback"]["compress_kernel_ms"], 2)
+    r["tma_vs_scalar_speedup"] = round(r["load_scalar_per_thread"]["compress_kernel_ms"] / r["decoupled_lookback"]["compress_kernel_ms"], 2)
     # random access on the Outlier stream
     cz.compress(x, lam, spec.eb_mode, "outlier", out=out, out_bytes=nb)
     y = torch.empty(1 << 20, dtype=x.dtype, device="cuda")
@@ -49,6 +54,13 @@ for cfg in sys.argv[1:] or ["cfg3b", "cfg5"]:
     yfull = torch.empty_like(x)
     t = timeit(lambda: cz.decompress(out, n, x.dtype, out=yfull), 5)
     ra["full_decompress_gbs"] = round(n * w / t / 1e9, 1)
+    scr = torch.empty(int(cz._lib.cszp2_decompress_scratch_bytes(n)), dtype=torch.uint8, device="cuda")
+    t_lb = timeit(lambda: cz.decompress_tilewise(out, n, x.dtype, cz.LOCATE_LOOKBACK, out=yfull, scratch=scr), 5)
+    t_ix = timeit(lambda: cz.decompress_tilewise(out, n, x.dtype, cz.LOCATE_INDEX, out=yfull, scratch=scr), 5)
+    r["decompress_locate"] = {
+        "persisted_index_persistent_kernel_gbs": ra["full_decompress_gbs"],
+        "persisted_index_cta_per_tile_gbs": round(n * w / t_ix / 1e9, 1),
+        "decompression_lookback_cta_per_tile_gbs": round(n * w / t_lb / 1e9, 1)}
     r["random_access"] = ra
     res[cfg] = r
     del x, out, yfull; torch.cuda.empty_cache()

@@ -297,3 +297,38 @@ def test_config5_single_gpu_sampled():
     _sampled_tile_parity(x, out, y, "outlier", sorted(set([0, T - 1] + list(rng.integers(0, T, 4)))))
     for s in range(0, n, 1 << 30):
         _error_bound_all(x[s:s + (1 << 30)], y[s:s + (1 << 30)], h["eb_abs"])
+
+
+@pytest.mark.parametrize("flags", [2, 4, 3, 5])
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_load_ablation_same_stream(flags, dtype):
+    """NEXT #2: per-thread vector / scalar loads (± chained scan) give the product stream."""
+    n = 7 * 8192 + 32 * 9 + 13
+    xh = make_field("cfg2", DEV, 0, n).cpu().numpy().astype(dtype)
+    x = torch.from_numpy(xh).to(DEV)
+    ref, rc = oracle.compress(xh, 1e-4, oracle.REL, oracle.OUTLIER)
+    out = torch.full((cz.compress_bound(n, x.dtype),), 0xAA, dtype=torch.uint8, device=DEV)
+    nb = torch.zeros(1, dtype=torch.int64, device=DEV)
+    cz.compress_prepare(x, 1e-4, "rel", out)
+    cz.compress_encode_ex(x, 1e-4, "rel", "outlier", out, nb, flags=flags)
+    torch.cuda.synchronize()
+    assert int(nb.item()) == ref.size
+    np.testing.assert_array_equal(out[: ref.size].cpu().numpy(), ref)
+
+
+@pytest.mark.parametrize("locate", [0, 1])
+@pytest.mark.parametrize("n", [0, 1, 8192, 5 * 8192 + 32 * 3 + 7])
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_decompress_tilewise_ablation(n, dtype, locate):
+    """NEXT #2: the paper-style decompression-side lookback decodes the same values."""
+    xh = make_field("cfg2", DEV, 0, max(n, 1)).cpu().numpy().astype(dtype)[:n]
+    ref, rc = oracle.compress(xh, 1e-4, oracle.REL, oracle.OUTLIER)
+    yr, rc = oracle.decompress(ref, n, dtype)
+    cmp = torch.from_numpy(ref).to(DEV)
+    st = torch.zeros(1, dtype=torch.int32, device=DEV)
+    y = cz.decompress_tilewise(cmp, n, torch.float32 if dtype == np.float32 else torch.float64, locate=locate,
+                               status=st)
+    torch.cuda.synchronize()
+    assert int(st.item()) == 0
+    iv = np.uint32 if dtype == np.float32 else np.uint64
+    np.testing.assert_array_equal(y.cpu().numpy().view(iv), yr.view(iv))
