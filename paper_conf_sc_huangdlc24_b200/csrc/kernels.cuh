@@ -685,7 +685,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
     __shared__ uint32_t s_qagg[NQ], s_qpos[NQ];
     __shared__ uint8_t s_qbad[NQ];
     __shared__ uint32_t s_warp[NT / 32];
-    __shared__ uint32_t s_pos, s_tkin;
+    __shared__ uint32_t s_tkin;
     __shared__ volatile uint32_t s_tail;  // ring bytes released by the resolver
     __shared__ volatile uint32_t s_end;   // queue index of the end marker
 
@@ -714,6 +714,19 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
             mbar_expect_tx(&s_full, 0);
         }
     };
+    // producer thread 0: publish the claimed ticket, then arrive on s_full (with the
+    // TMA bytes, or without data past the last tile): the mbarrier's release/acquire
+    // makes s_tkin visible to the producers waiting on s_full, so no extra barrier
+    auto claim = [&](uint32_t tk) {
+        s_tkin = tk;
+        if (tk < T_eff) {
+            TRACE(tk, 0, gtimer());
+            TRACE(tk, 7, blockIdx.x);
+            issue(tk);
+        } else {
+            mbar_expect_tx(&s_full, 0);
+        }
+    };
 
     if (tid == 0) {
         s_end = 0xFFFFFFFFu;
@@ -724,13 +737,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
             mbar_init(&s_done[i], 1);
         }
         fence_mbar_init();
-        const uint32_t tk = atomicAdd(ticket, 1u);
-        s_tkin = tk;
-        if (tk < T_eff) {
-            TRACE(tk, 0, gtimer());
-            TRACE(tk, 7, blockIdx.x);
-            issue(tk);
-        }
+        claim(atomicAdd(ticket, 1u));
     }
     __syncthreads();
 
@@ -740,7 +747,12 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
         uint32_t head = 0, last_agg = 0;  // ring allocation cursor, latest payload (thread 0)
         for (uint32_t it = 0;; ++it) {
             const int q = it % NQ;
-            const uint64_t t = s_tkin;  // visible: barrier at the end of the previous iteration
+            // claim the next tile now if the ring clearly has room for two more payloads
+            uint32_t tk_next = 0;
+            const bool ahead = (tid == 0) && (head - s_tail + 2 * last_agg + 64 <= LY::RING);
+            if (ahead) tk_next = atomicAdd(ticket, 1u);  // consumed after the buffer is free
+            mbar_wait(&s_full, it & 1);
+            const uint64_t t = s_tkin;  // published before the arrival we just waited for
             if (t >= T_eff) {           // end marker for the resolver
                 if (tid == 0) {
                     if (it >= NQ) mbar_wait(&s_done[q], (it / NQ - 1) & 1);
@@ -749,11 +761,6 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
                 }
                 break;
             }
-            // claim the next tile now if the ring clearly has room for two more payloads
-            uint32_t tk_next = 0;
-            const bool ahead = (tid == 0) && (head - s_tail + 2 * last_agg + 64 <= LY::RING);
-            if (ahead) tk_next = atomicAdd(ticket, 1u);  // consumed after the buffer is free
-            mbar_wait(&s_full, it & 1);
             if (tid == 0) TRACE(t, 1, gtimer());
             const uint64_t b = t * BPT + tid;
             const bool active = b < g.nb;
@@ -821,42 +828,27 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
 
             // the input buffer is free after this barrier: start the next tile's load
             const bool any_bad = named_sync_or(BAR_PROD, NT, bad);
-            if (ahead) {
-                s_tkin = tk_next;
-                if (tk_next < T_eff) {
-                    TRACE(tk_next, 0, gtimer());
-                    TRACE(tk_next, 7, blockIdx.x);
-                    issue(tk_next);
-                }
-            }
+            if (ahead) claim(tk_next);
             // intra-tile scan ("Reduce")
             uint32_t agg;
             const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg, BAR_PROD);
-            if (tid == 0) {
-                if (g.T) publish_aggregate(index, t, agg, any_bad);
-                TRACE(t, 2, gtimer());
-                // ring space (16-aligned, contiguous) and a queue slot
-                uint32_t pos = (head + 15u) & ~15u;
-                if ((pos % LY::RING) + agg > LY::RING) pos = (pos / LY::RING + 1) * LY::RING;
-                // wait for room; an empty ring always has room (a payload that had to skip
-                // the ring's end can then never find the skipped bytes still "in use")
-                while (pos + agg > s_tail + LY::RING && s_tail != head) __nanosleep(64);
-                head = pos + agg;
-                last_agg = agg;
-                if (it >= NQ) mbar_wait(&s_done[q], (it / NQ - 1) & 1);
-                s_pos = pos;
-                s_qt[q] = t;
-                s_qagg[q] = agg;
-                s_qbad[q] = any_bad;
-                s_qpos[q] = pos;
-            }
+            if (tid == 0 && g.T) publish_aggregate(index, t, agg, any_bad);
+            if (tid == 0) TRACE(t, 2, gtimer());
+            // ring space (16-aligned, contiguous), computed identically by every producer
+            // thread from (head, agg); each waits for room itself. An empty ring always has
+            // room (a payload that had to skip the ring's end can then never find the
+            // skipped bytes still "in use").
+            uint32_t pos = (head + 15u) & ~15u;
+            if ((pos % LY::RING) + agg > LY::RING) pos = (pos / LY::RING + 1) * LY::RING;
+            while (pos + agg > s_tail + LY::RING && s_tail != head) __nanosleep(64);
+            head = pos + agg;
+            last_agg = agg;
             if (active) out[g.O + b] = static_cast<uint8_t>(obyte);  // ❹ offset bytes
-            named_sync(BAR_PROD, NT);  // s_pos visible
 
             // ❷ payload staged in the ring at its tile-relative byte offset; bit planes
             // by an in-register transpose sized to the warp's largest fixed length
             {
-                const uint32_t st = (s_pos % LY::RING) + my_excl;
+                const uint32_t st = (pos % LY::RING) + my_excl;
                 const uint32_t outl = a[0];
                 if (OUTLIER && nob) a[0] = 0;  // the outlier slot of every plane is 0
                 const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, static_cast<unsigned>(size ? fl : 0)));
@@ -887,19 +879,17 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
             named_sync(BAR_PROD, NT);  // staging complete
             if (tid == 0) {
                 TRACE(t, 4, gtimer());
+                if (it >= NQ) mbar_wait(&s_done[q], (it / NQ - 1) & 1);  // queue slot free
+                s_qt[q] = t;
+                s_qagg[q] = agg;
+                s_qbad[q] = any_bad;
+                s_qpos[q] = pos;
                 mbar_arrive(&s_staged[q]);
                 if (!ahead) {  // claim now, nothing unpublished held: wait for ring room first
                     while (head - s_tail + 2 * last_agg + 64 > LY::RING && head != s_tail) __nanosleep(64);
-                    const uint32_t tk = atomicAdd(ticket, 1u);
-                    s_tkin = tk;
-                    if (tk < T_eff) {
-                        TRACE(tk, 0, gtimer());
-                        TRACE(tk, 7, blockIdx.x);
-                        issue(tk);
-                    }
+                    claim(atomicAdd(ticket, 1u));
                 }
             }
-            named_sync(BAR_PROD, NT);  // s_tkin visible
         }
     } else {
         // ============================== resolver: ❸ then ❹, in tile order
