@@ -30,7 +30,7 @@ __device__ __forceinline__ uint64_t gtimer() {
     return t;
 }
 #define TRACE(tile, slot, val) \
-    do { if (g_trace) g_trace[(tile) * 8 + (slot)] = (val); } while (0)
+    do { if (g_trace) g_trace[(tile) * 16 + (slot)] = (val); } while (0)
 #else
 #define TRACE(tile, slot, val) do { } while (0)
 #endif
@@ -378,67 +378,63 @@ struct LookbackWindow {
     uint64_t d[LB_PER_LANE];
 };
 
+// Window rows: row u, lane l holds the descriptor of tile j − (32u + l) (nearest first;
+// each row is one coalesced 256-byte load).
 __device__ __forceinline__ void lookback_issue(const uint64_t *index, int64_t j, LookbackWindow &w) {
-    const int64_t base = j - (threadIdx.x & 31) * LB_PER_LANE;
+    const int64_t base = j - (threadIdx.x & 31);
 #pragma unroll
     for (int u = 0; u < LB_PER_LANE; u++)
-        w.d[u] = (base - u >= 0) ? ld_relaxed_u64(&index[base - u]) : FLAG_P;  // virtual P|0
+        w.d[u] = (base - 32 * u >= 0) ? ld_relaxed_u64(&index[base - 32 * u]) : FLAG_P;  // virtual P|0
 }
 
 // Returns the exclusive prefix of tile t (>= 1) and publishes its inclusive
-// descriptor; *range_out = RANGE bit of the inclusive prefix.
+// descriptor; *range_out = RANGE bit of the inclusive prefix. Row by row, nearest
+// first: the first P in the row ends the walk; every slot before it must be A (a
+// Waiting one is re-polled); A values (tile aggregates < 2^32) are summed with one
+// warp reduction per row.
 __device__ __forceinline__ uint64_t lookback_finish(uint64_t *index, uint64_t t, uint64_t agg,
                                                     bool bad, LookbackWindow &w, bool *range_out) {
     const int lane = threadIdx.x & 31;
-    uint64_t excl = 0, rbits = bad ? BIT_RANGE : 0;
+    uint64_t excl = 0;
+    bool rb = bad;
     int64_t j = static_cast<int64_t>(t) - 1;  // nearest predecessor of the window
-    bool done = false;
-    while (!done) {
-        const int64_t base = j - lane * LB_PER_LANE;
-        while (true) {
-            // lane-local walk, nearest first: st 2 = met a P, 1 = all A, 0 = met a Waiting slot
-            uint64_t sum = 0, rb = 0;
-            int st = 1;
+    while (true) {
+        bool done = false;
 #pragma unroll
-            for (int u = 0; u < LB_PER_LANE; u++) {
-                if (st == 1) {
-                    const uint64_t f = w.d[u] >> 62;
-                    if (f == 0) {
-                        st = 0;
-                    } else {
-                        sum += w.d[u] & VAL61;
-                        rb |= w.d[u] & BIT_RANGE;
-                        if (f == 2) st = 2;
-                    }
+        for (int u = 0; u < LB_PER_LANE; u++) {
+            if (!done) {
+                uint64_t d = w.d[u];
+                unsigned pm = __ballot_sync(0xffffffffu, (d >> 62) == 2);
+                unsigned wm = __ballot_sync(0xffffffffu, (d >> 62) == 0);
+                int p = pm ? __ffs(pm) - 1 : 32;
+                while (wm && __ffs(wm) - 1 < p) {  // a needed predecessor is still Waiting
+#ifdef CSZP2_TRACE
+                    if (lane == 0 && g_trace) g_trace[t * 16 + 5]++;
+#endif
+                    __nanosleep(32);
+                    const int64_t idx = j - 32 * u - lane;
+                    if ((d >> 62) == 0 && idx >= 0) d = ld_relaxed_u64(&index[idx]);
+                    pm = __ballot_sync(0xffffffffu, (d >> 62) == 2);
+                    wm = __ballot_sync(0xffffffffu, (d >> 62) == 0);
+                    p = pm ? __ffs(pm) - 1 : 32;
+                }
+                excl += __reduce_add_sync(0xffffffffu, lane < p ? static_cast<uint32_t>(d & VAL61) : 0u);
+                rb |= __ballot_sync(0xffffffffu, lane <= p && (d & BIT_RANGE)) != 0;
+                if (p < 32) {
+                    excl += __shfl_sync(0xffffffffu, d & VAL61, p);
+                    done = true;
                 }
             }
-            const unsigned pm = __ballot_sync(0xffffffffu, st == 2);
-            const unsigned wm = __ballot_sync(0xffffffffu, st == 0);
-            const int p = pm ? __ffs(pm) - 1 : 32;
-            const int wt = wm ? __ffs(wm) - 1 : 32;
-            if (wt < p) {  // a needed predecessor is still Waiting: re-poll the empty slots
+        }
+        if (done) break;
 #ifdef CSZP2_TRACE
-                if (lane == 0 && g_trace) g_trace[t * 8 + 5]++;
+        if (lane == 0 && g_trace) g_trace[t * 16 + 5] += 1ll << 32;  // extra window
 #endif
-                __nanosleep(32);
-#pragma unroll
-                for (int u = 0; u < LB_PER_LANE; u++)
-                    if (base - u >= 0 && (w.d[u] >> 62) == 0) w.d[u] = ld_relaxed_u64(&index[base - u]);
-                continue;
-            }
-            excl += warp_sum_u64(lane <= p ? sum : 0);
-            rbits |= __ballot_sync(0xffffffffu, lane <= p && rb != 0) ? BIT_RANGE : 0;
-            done = p < 32;
-            break;
-        }
-        if (!done) {
-
-            j -= 32 * LB_PER_LANE;
-            lookback_issue(index, j, w);
-        }
+        j -= 32 * LB_PER_LANE;
+        lookback_issue(index, j, w);
     }
-    if (lane == 0) st_relaxed_u64(&index[t], FLAG_P | rbits | (excl + agg));
-    *range_out = rbits != 0;
+    if (lane == 0) st_relaxed_u64(&index[t], FLAG_P | (rb ? BIT_RANGE : 0) | (excl + agg));
+    *range_out = rb;
     return excl;
 }
 
@@ -905,8 +901,10 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
             if (lane == 0) TRACE(t, 6, gtimer());
             bool rng = bad;
             uint64_t excl = 0;
+            const bool chained = (hs.flags & 1u) != 0;
+            if (lane == 0) TRACE(t, 8, gtimer());
             if (g.T && t > 0) {
-                if (hs.flags & 1u)  // ablation: plain chained scan (Fig 12 left)
+                if (chained)  // ablation: plain chained scan (Fig 12 left)
                     excl = chained_prefix(index, t, agg, bad, &rng);
                 else
                     excl = lookback(index, t, agg, bad, &rng);
@@ -914,6 +912,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
             if (lane == 0) TRACE(t, 3, gtimer());
             const uint64_t dst0 = g.D + excl;
             write_payload(ring + (pos % LY::RING), out, dst0, agg, lane, 32);
+            if (lane == 0) TRACE(t, 9, gtimer());
             if (t == T_eff - 1) {  // last tile: pads, header, d_out_bytes
                 const uint64_t dst1 = dst0 + agg;
                 __syncwarp();

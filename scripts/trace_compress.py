@@ -15,17 +15,19 @@ for arg in sys.argv[1:]:
     x = make_field(cfg, "cuda"); n = x.numel()
     T = -(-(-(-n // 32)) // 256)
     out = torch.empty(lib.cszp2_compress_bound(n, 0), dtype=torch.uint8, device="cuda")
-    tr = torch.zeros(T * 8, dtype=torch.int64, device="cuda")
+    tr = torch.zeros(T * 16, dtype=torch.int64, device="cuda")
     lib.cszp2_debug_set_trace(ctypes.c_void_p(tr.data_ptr()))
     st = torch.cuda.current_stream().cuda_stream
     for rep in range(3):
         tr.zero_()
         lib.cszp2_compress(ctypes.c_void_p(x.data_ptr()), n, 0, spec.ebs[-1], 1, enc, ctypes.c_void_p(out.data_ptr()), None, ctypes.c_void_p(st))
         torch.cuda.synchronize()
-    a = tr.view(T, 8).cpu().numpy().astype(np.int64)
+    a = tr.view(T, 16).cpu().numpy().astype(np.int64)
     t0 = a[:, 0][a[:, 0] > 0].min()
     a[:, :5] -= t0
     a[:, 6] -= t0
+    a[:, 8] -= t0
+    a[:, 9] -= t0
     claim, data, pub, res, staged, polls, rstart = [a[:, i] for i in range(7)]
     moves = np.zeros_like(polls)
     print(f"== {cfg}: T={T} span={(res.max())/1e3:.1f}us rate={T/(res.max()/1e3):.1f} tiles/us")
@@ -37,8 +39,20 @@ for arg in sys.argv[1:]:
     print("pubA->resolved", q((res[1:]-pub[1:])/1e3))
     print("staged->rstart", q((rstart[1:]-staged[1:])/1e3))
     print("rstart->resolved", q((res[1:]-rstart[1:])/1e3))
+    issued, copied = a[:, 8], a[:, 9]
+    print("rstart->issued", q((issued[1:]-rstart[1:])/1e3))
+    print("issued->resolved", q((res[1:]-issued[1:])/1e3))
+    print("resolved->copied", q((copied[1:]-res[1:])/1e3))
     print("claim->resolved", q((res[1:]-claim[1:])/1e3))
-    print("polls mean", polls.mean(), "max", polls.max(), "moves mean", moves.mean())
+    windows = 1 + (polls >> 32)
+    polls = polls & 0xFFFFFFFF
+    print("polls mean", polls.mean(), "max", polls.max(), "windows mean", windows.mean(), "pct", q(windows))
+    # distance from a tile to the previous tile of the same CTA (slot 7 = CTA id)
+    cta_ = a[:, 7]
+    o = np.lexsort((np.arange(T), cta_))
+    same = cta_[o][1:] == cta_[o][:-1]
+    dist = (o[1:] - o[:-1])[same]
+    print("distance to the same CTA's previous tile", q(dist))
     # frontier: resolved time vs tile index; claim order vs time
     order = np.argsort(claim)
     print("claims per us (median over 10us windows):", np.median(np.diff(np.searchsorted(np.sort(claim), np.arange(0, claim.max(), 10000))))/10)
