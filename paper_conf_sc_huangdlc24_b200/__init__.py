@@ -15,6 +15,9 @@ import torch
 
 from ._build import LIB as _LIB_PATH
 
+# dev aid (scripts/ab_libs.py): load another build of the same C ABI for A/B timing
+_LIB_PATH = os.environ.get("CSZP2_LIB", _LIB_PATH)
+
 F32, F64 = 0, 1
 EB_ABS, EB_REL = 0, 1
 ENC_PLAIN, ENC_OUTLIER = 0, 1

@@ -108,6 +108,39 @@ __device__ __forceinline__ int quantize(double x, double inv, bool &bad) {
     bad |= !(fabs(t) <= 1073741823.0);
     return __double2int_rn(t);
 }
+// Whole-block ❶ for the 1D compressor, bit-identical to quantize() above but without the
+// slow F2I conversions (1/8-rate pipe) in the common case: for |t| < 2^22,
+// fl(t + 1.5·2^23) lies in [2^23, 2^24) where the float spacing is 1, so the RN addition
+// rounds t half-to-even to an integer that is read straight out of the bit pattern.
+// A block with any |t| >= 2^22 (or NaN) takes the F2I path with the full range check.
+// (f64: fl(t + 1.5·2^52) does the same for every |t| < 2^51, the low word is rint(t).)
+__device__ __forceinline__ void quantize_block(const float (&x)[L], float inv, int (&q)[L], bool &bad) {
+    float t[L];
+    bool big = false;
+#pragma unroll
+    for (int i = 0; i < L; i++) {
+        t[i] = __fmul_rn(x[i], inv);
+        big |= !(fabsf(t[i]) < 4194304.0f);
+    }
+    if (!big) {
+#pragma unroll
+        for (int i = 0; i < L; i++) q[i] = __float_as_int(__fadd_rn(t[i], 12582912.0f)) - 0x4B400000;
+    } else {
+#pragma unroll
+        for (int i = 0; i < L; i++) {
+            bad |= !(fabsf(t[i]) <= 1073741760.0f);
+            q[i] = __float2int_rn(t[i]);
+        }
+    }
+}
+__device__ __forceinline__ void quantize_block(const double (&x)[L], double inv, int (&q)[L], bool &bad) {
+#pragma unroll
+    for (int i = 0; i < L; i++) {
+        const double t = __dmul_rn(x[i], inv);
+        bad |= !(fabs(t) <= 1073741823.0);
+        q[i] = static_cast<int>(static_cast<uint32_t>(__double_as_longlong(__dadd_rn(t, 6755399441055744.0))));
+    }
+}
 __device__ __forceinline__ float dequantize(int q, float s) { return __fmul_rn(__int2float_rn(q), s); }
 __device__ __forceinline__ double dequantize(int q, double s) {
     return __dmul_rn(__int2double_rn(q), s);
@@ -388,10 +421,12 @@ __device__ __forceinline__ void lookback_issue(const uint64_t *index, int64_t j,
 }
 
 // Returns the exclusive prefix of tile t (>= 1) and publishes its inclusive
-// descriptor; *range_out = RANGE bit of the inclusive prefix. Row by row, nearest
-// first: the first P in the row ends the walk; every slot before it must be A (a
-// Waiting one is re-polled); A values (tile aggregates < 2^32) are summed with one
-// warp reduction per row.
+// descriptor; *range_out = RANGE bit of the inclusive prefix. Slot (row u, lane l) has
+// the nearest-first key 32u + l. Per window, a constant number of warp collectives
+// (not one set per row): the nearest P and the nearest Waiting slot by two min
+// reductions; if a Waiting slot is nearer than the P, the Waiting slots are re-polled;
+// otherwise every slot before the P is an A, whose values (tile aggregates, each
+// <= 256 * 132 bytes, so 256 of them fit in 32 bits) are summed by one reduction.
 __device__ __forceinline__ uint64_t lookback_finish(uint64_t *index, uint64_t t, uint64_t agg,
                                                     bool bad, LookbackWindow &w, bool *range_out) {
     const int lane = threadIdx.x & 31;
@@ -399,34 +434,44 @@ __device__ __forceinline__ uint64_t lookback_finish(uint64_t *index, uint64_t t,
     bool rb = bad;
     int64_t j = static_cast<int64_t>(t) - 1;  // nearest predecessor of the window
     while (true) {
-        bool done = false;
+        uint32_t pk = 0xFFFFu, wk = 0xFFFFu;
+#pragma unroll
+        for (int u = LB_PER_LANE - 1; u >= 0; u--) {  // descending: the nearest row wins
+            const uint32_t f = static_cast<uint32_t>(w.d[u] >> 62);
+            if (f == 2) pk = 32u * u + lane;
+            if (f == 0) wk = 32u * u + lane;
+        }
+        const uint32_t P = __reduce_min_sync(0xffffffffu, pk);
+        const uint32_t W = __reduce_min_sync(0xffffffffu, wk);
+        if (W < P) {  // a needed predecessor is still Waiting: re-poll the Waiting slots
+#ifdef CSZP2_TRACE
+            if (lane == 0 && g_trace) g_trace[t * 16 + 5]++;
+#endif
+            __nanosleep(32);
+#pragma unroll
+            for (int u = 0; u < LB_PER_LANE; u++) {
+                const int64_t idx = j - 32 * u - lane;
+                if ((w.d[u] >> 62) == 0 && idx >= 0) w.d[u] = ld_relaxed_u64(&index[idx]);
+            }
+            continue;
+        }
+        uint32_t s = 0;
+        bool r = false;
+        uint64_t pv = 0;
 #pragma unroll
         for (int u = 0; u < LB_PER_LANE; u++) {
-            if (!done) {
-                uint64_t d = w.d[u];
-                unsigned pm = __ballot_sync(0xffffffffu, (d >> 62) == 2);
-                unsigned wm = __ballot_sync(0xffffffffu, (d >> 62) == 0);
-                int p = pm ? __ffs(pm) - 1 : 32;
-                while (wm && __ffs(wm) - 1 < p) {  // a needed predecessor is still Waiting
-#ifdef CSZP2_TRACE
-                    if (lane == 0 && g_trace) g_trace[t * 16 + 5]++;
-#endif
-                    __nanosleep(32);
-                    const int64_t idx = j - 32 * u - lane;
-                    if ((d >> 62) == 0 && idx >= 0) d = ld_relaxed_u64(&index[idx]);
-                    pm = __ballot_sync(0xffffffffu, (d >> 62) == 2);
-                    wm = __ballot_sync(0xffffffffu, (d >> 62) == 0);
-                    p = pm ? __ffs(pm) - 1 : 32;
-                }
-                excl += __reduce_add_sync(0xffffffffu, lane < p ? static_cast<uint32_t>(d & VAL61) : 0u);
-                rb |= __ballot_sync(0xffffffffu, lane <= p && (d & BIT_RANGE)) != 0;
-                if (p < 32) {
-                    excl += __shfl_sync(0xffffffffu, d & VAL61, p);
-                    done = true;
-                }
-            }
+            const uint32_t key = 32u * u + lane;
+            const uint64_t d = w.d[u];
+            if (key < P) s += static_cast<uint32_t>(d);  // an A: value < 2^32
+            if (key <= P) r |= (d & BIT_RANGE) != 0;
+            if (key == P) pv = d & VAL61;
         }
-        if (done) break;
+        excl += __reduce_add_sync(0xffffffffu, s);
+        rb |= __any_sync(0xffffffffu, r);
+        if (P < 32u * LB_PER_LANE) {
+            excl += __shfl_sync(0xffffffffu, pv, P & 31u);
+            break;
+        }
 #ifdef CSZP2_TRACE
         if (lane == 0 && g_trace) g_trace[t * 16 + 5] += 1ll << 32;  // extra window
 #endif
@@ -682,6 +727,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
     __shared__ uint8_t s_qbad[NQ];
     __shared__ uint32_t s_warp[NT / 32];
     __shared__ uint32_t s_tkin;
+    __shared__ uint64_t s_rel;            // producer warps done reading the input buffer
     __shared__ volatile uint32_t s_tail;  // ring bytes released by the resolver
     __shared__ volatile uint32_t s_end;   // queue index of the end marker
 
@@ -727,6 +773,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
     if (tid == 0) {
         s_end = 0xFFFFFFFFu;
         s_tail = 0;
+        mbar_init(&s_rel, NT / 32);
         mbar_init(&s_full, 1);
         for (int i = 0; i < NQ; i++) {
             mbar_init(&s_staged[i], 1);
@@ -740,13 +787,19 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
     if (warp < RESOLVE_WARP) {
         // ============================== producers
         const auto K = make_consts(eb_abs, static_cast<T *>(nullptr));
-        uint32_t head = 0, last_agg = 0;  // ring allocation cursor, latest payload (thread 0)
+        // ring allocation cursor and latest payload size: identical in every producer thread
+        uint32_t head = 0, last_agg = 0;
         for (uint32_t it = 0;; ++it) {
             const int q = it % NQ;
-            // claim the next tile now if the ring clearly has room for two more payloads
+            // thread 0 takes the next ticket while the data is in flight (if the ring
+            // clearly has room for two more payloads); the atomic's result stays in a
+            // register until the buffer is released, so nothing waits on its round trip
             uint32_t tk_next = 0;
-            const bool ahead = (tid == 0) && (head - s_tail + 2 * last_agg + 64 <= LY::RING);
-            if (ahead) tk_next = atomicAdd(ticket, 1u);  // consumed after the buffer is free
+            bool ahead = false;
+            if (tid == 0) {
+                ahead = head - s_tail + 2 * last_agg + 64 <= LY::RING;
+                if (ahead) tk_next = atomicAdd(ticket, 1u);
+            }
             mbar_wait(&s_full, it & 1);
             const uint64_t t = s_tkin;  // published before the arrival we just waited for
             if (t >= T_eff) {           // end marker for the resolver
@@ -780,11 +833,21 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
                 for (int i = 0; i < L; i++) x[i] = (i < (int)valid) ? in[b * L + i] : T(0);
             }
 
+            // The input buffer is free once every producer warp holds its values in
+            // registers (s_rel: one arrival per warp): warp 0 then issues the TMA load of
+            // the tile taken ahead (otherwise thread 0 claims after staging), so the load
+            // overlaps this tile's whole encode; the other warps go straight on.
+            __syncwarp();
+            if ((tid & 31) == 0) mbar_arrive(&s_rel);
+            if (warp == 0) {
+                mbar_wait(&s_rel, it & 1);
+                if (ahead) claim(tk_next);
+            }
+
             // ❶ pre-quantization + in-block first-order difference
             bool bad = false;
             int qv[L];
-#pragma unroll
-            for (int i = 0; i < L; i++) qv[i] = quantize(x[i], K.inv, bad);
+            quantize_block(x, K.inv, qv, bad);
             if (!full) {  // tail block: q_i = q_{i-1} past n (FORMAT.md §6.4)
 #pragma unroll
                 for (int i = 1; i < L; i++)
@@ -822,9 +885,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
             }
             if (!K.ok) bad = true;
 
-            // the input buffer is free after this barrier: start the next tile's load
             const bool any_bad = named_sync_or(BAR_PROD, NT, bad);
-            if (ahead) claim(tk_next);
             // intra-tile scan ("Reduce")
             uint32_t agg;
             const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg, BAR_PROD);

@@ -3,7 +3,7 @@ import sys, os, ctypes
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
 from synthetic import CONFIGS, make_field
-lib = ctypes.CDLL(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "paper_conf_sc_huangdlc24_b200", "libcszp2_trace.so"))
+lib = ctypes.CDLL(os.environ.get("CSZP2_TRACE_LIB", os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "paper_conf_sc_huangdlc24_b200", "libcszp2_trace.so")))
 vp, u64, i32, dbl = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int, ctypes.c_double
 lib.cszp2_compress.argtypes = [vp, u64, i32, dbl, i32, i32, vp, vp, vp]
 lib.cszp2_compress_bound.argtypes = [u64, i32]; lib.cszp2_compress_bound.restype = u64
@@ -75,3 +75,20 @@ for arg in sys.argv[1:]:
     print(f"per-CTA period {np.median(per)/1e3:.2f}us  staged->next data {np.median(waits)/1e3:.2f}us  compute {np.median(comp)/1e3:.2f}us  staging {np.median(stg)/1e3:.2f}us")
     w = np.array([x for x in waits])
     print("staged->next data pct", q(w/1e3))
+    # tails: per CTA, consecutive data arrivals; where do the long gaps come from?
+    gaps = []; parts = []
+    for c in np.unique(cta):
+        idx = np.where(cta == c)[0]
+        idx = idx[np.argsort(data[idx])]
+        if len(idx) < 3: continue
+        g = np.diff(data[idx])
+        gaps.append(g)
+        # for tile k+1: claim(k+1) - data(k), data(k+1) - claim(k+1), staged(k) - data(k)
+        parts.append(np.stack([g, claim[idx][1:] - data[idx][:-1], data[idx][1:] - claim[idx][1:],
+                               staged[idx][:-1] - data[idx][:-1]], 1))
+    G = np.concatenate(gaps); Pm = np.concatenate(parts)
+    print(f"period mean {G.mean()/1e3:.3f}us median {np.median(G)/1e3:.3f}us  pct", q(G/1e3))
+    big = Pm[:, 0] > 2 * np.median(G)
+    print(f"long gaps (>2x median): {big.mean()*100:.2f}% of tiles, {Pm[big,0].sum()/G.sum()*100:.1f}% of time; "
+          f"mean [gap, data->claim(next), claim->data(next), data->staged] = {np.round(Pm[big].mean(0)/1e3, 2)} us")
+    print(f"all tiles mean [gap, data->claim(next), claim->data(next), data->staged] = {np.round(Pm.mean(0)/1e3, 2)} us")
