@@ -118,6 +118,23 @@ int check_compress_args(const void *d_in, uint64_t n, int dtype, double eb, int 
 template <typename T>
 int launch_minmax(const void *d_in, uint64_t n, double lambda, void *d_out, cudaStream_t st) {
     const int sms = sm_count();
+    const uint64_t nchunks = n * sizeof(T) / MM_CHUNK;
+    if (nchunks >= static_cast<uint64_t>(sms)) {  // bulk-TMA streaming, 2 CTAs per SM
+        constexpr int smem = MM_STAGES * MM_CHUNK;
+        static std::once_flag once;
+        static int attr_rc = CSZP2_OK;
+        std::call_once(once, [] {
+            if (cudaFuncSetAttribute(minmax_kernel_tma<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     smem) != cudaSuccess)
+                attr_rc = CSZP2_ERR_CUDA;
+        });
+        if (attr_rc != CSZP2_OK) return attr_rc;
+        const uint64_t want = 2ull * sms;
+        const int grid = static_cast<int>(nchunks < want ? nchunks : want);
+        minmax_kernel_tma<T><<<grid, 256, smem, st>>>(static_cast<const T *>(d_in), n, lambda,
+                                                       static_cast<uint8_t *>(d_out));
+        return launch_status();
+    }
     const uint64_t nvec = n / (16 / sizeof(T));
     uint64_t want = (nvec + 255) / 256;
     int grid = static_cast<int>(want < 1 ? 1 : (want > (uint64_t)sms * 8 ? (uint64_t)sms * 8 : want));

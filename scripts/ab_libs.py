@@ -29,19 +29,20 @@ for cfg in sys.argv[1].split(","):
     y = torch.empty_like(x)
     lam = spec.ebs[-1]
     for enc in ("outlier", "plain"):
-        te, td = [], []
+        te, td, tp = [], [], []
         for it in range(8):
-            cz.compress_prepare(x, lam, spec.eb_mode, out)
+            s0, e0 = torch.cuda.Event(True), torch.cuda.Event(True)
+            s0.record(); cz.compress_prepare(x, lam, spec.eb_mode, out); e0.record()
             s, e = torch.cuda.Event(True), torch.cuda.Event(True)
             s.record(); cz.compress_encode(x, lam, spec.eb_mode, enc, out, nb); e.record()
             s2, e2 = torch.cuda.Event(True), torch.cuda.Event(True)
             s2.record(); cz.decompress(out, n, x.dtype, out=y); e2.record()
             torch.cuda.synchronize()
             if it >= 3:
-                te.append(s.elapsed_time(e)); td.append(s2.elapsed_time(e2))
+                te.append(s.elapsed_time(e)); td.append(s2.elapsed_time(e2)); tp.append(s0.elapsed_time(e0))
         tot = int(nb.item())
-        te.sort(); td.sort()
-        res[f"{cfg}/{enc}"] = dict(cr=round(n * w / tot, 2), enc_ms=te[len(te)//2], dec_ms=td[len(td)//2],
+        te.sort(); td.sort(); tp.sort()
+        res[f"{cfg}/{enc}"] = dict(prep_gbs=round(n * w / tp[len(tp)//2] / 1e6, 1), cr=round(n * w / tot, 2), enc_ms=te[len(te)//2], dec_ms=td[len(td)//2],
                                    enc_gbs=round((n * w + tot) / te[len(te)//2] / 1e6, 1),
                                    dec_gbs=round((n * w + tot) / td[len(td)//2] / 1e6, 1))
     del x, out, y
