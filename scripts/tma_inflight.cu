@@ -123,6 +123,36 @@ __global__ void __launch_bounds__(256) stream_kernel(const __grid_constant__ CUt
     if (acc == 0x12345678u) atomicAdd(sink, 1ull);
 }
 
+// write side: CTAs bulk-store a 32 KiB shared buffer to consecutive tiles, K groups in flight
+__global__ void __launch_bounds__(256) store_kernel(uint8_t *out, unsigned ntiles, int K, int D, unsigned *ticket) {
+    extern __shared__ uint8_t raw[];
+    uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(raw) + 1023) & ~uintptr_t(1023));
+    __shared__ unsigned s_t;
+    for (int i = threadIdx.x; i < (int)(TILE / 4); i += blockDim.x) reinterpret_cast<uint32_t *>(buf)[i] = i;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    __syncthreads();
+    while (true) {
+        if (threadIdx.x == 0) s_t = atomicAdd(ticket, 1u);
+        __syncthreads();
+        const unsigned t = s_t;
+        __syncthreads();
+        if (t >= ntiles) break;
+        if (threadIdx.x == 0) {
+            asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(out + (uint64_t)t * TILE),
+                         "r"(smem_u32(buf)), "r"(TILE) : "memory");
+            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+            if (K <= 1) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+            else if (K == 2) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+            else asm volatile("cp.async.bulk.wait_group.read 3;" ::: "memory");
+        }
+        if (D > 0) {
+            const uint64_t t0 = gtimer();
+            while (gtimer() - t0 < (uint64_t)D) {}
+        }
+    }
+    if (threadIdx.x == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+}
+
 int main(int argc, char **argv) {
     const uint64_t bytes = (argc > 1 ? strtoull(argv[1], 0, 0) : (8ull << 30));
     const unsigned ntiles = (unsigned)(bytes / TILE);
@@ -154,6 +184,38 @@ int main(int argc, char **argv) {
     cudaEventCreate(&e0);
     cudaEventCreate(&e1);
     printf("bytes %.2f GiB, %d SMs\n", (double)ntiles * TILE / 1073741824.0, sms);
+    {
+        cudaFuncSetAttribute(store_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, TILE + 1024);
+        for (int C : {2, 3, 4, 6})
+            for (int K : {1, 2, 4})
+                for (int D : {0, 1500}) {
+                    float best = 1e9;
+                    for (int rep = 0; rep < 3; rep++) {
+                        cudaMemset(ticket, 0, 4);
+                        cudaEventRecord(e0);
+                        store_kernel<<<sms * C, 256, TILE + 1024>>>(in, ntiles, K, D, ticket);
+                        cudaEventRecord(e1);
+                        cudaEventSynchronize(e1);
+                        float ms;
+                        cudaEventElapsedTime(&ms, e0, e1);
+                        if (ms < best) best = ms;
+                    }
+                    printf("store     C=%d K=%d D=%4d ns: %7.1f GB/s %s\n", C, K, D, (double)ntiles * TILE / best / 1e6,
+                           cudaGetErrorString(cudaGetLastError()));
+                }
+        float best = 1e9;
+        for (int rep = 0; rep < 3; rep++) {
+            cudaEventRecord(e0);
+            cudaMemsetAsync(in, rep, (uint64_t)ntiles * TILE);
+            cudaEventRecord(e1);
+            cudaEventSynchronize(e1);
+            float ms;
+            cudaEventElapsedTime(&ms, e0, e1);
+            if (ms < best) best = ms;
+        }
+        printf("cudaMemset: %7.1f GB/s\n", (double)ntiles * TILE / best / 1e6);
+        if (argc > 2) return 0;
+    }
     const char *names[] = {"bulk32K", "bulk8x4K", "tensor2D", "cp.async16", "ldg16"};
     const int CK[][2] = {{3, 1}, {3, 2}, {2, 2}, {2, 3}, {4, 1}, {6, 1}};
     const int Ds[] = {0, 1500};
