@@ -113,37 +113,55 @@ __device__ __forceinline__ int quantize(double x, double inv, bool &bad) {
 // fl(t + 1.5·2^23) lies in [2^23, 2^24) where the float spacing is 1, so the RN addition
 // rounds t half-to-even to an integer that is read straight out of the bit pattern.
 // A block with any |t| >= 2^22 (or NaN) takes the F2I path with the full range check.
-// (f64: fl(t + 1.5·2^52) does the same for every |t| < 2^51, the low word is rint(t).)
-__device__ __forceinline__ void quantize_block(const float (&x)[L], float inv, int (&q)[L], bool &bad) {
-    float t[L];
-    bool big = false;
+// Output is BIASED: qb_i = q_i + QBIAS (mod 2^32), so that the bit patterns can be
+// differenced directly (d_i = qb_i - qb_{i-1}, q_{-1} = 0 <=> qb_{-1} = QBIAS).
+// (f64: fl(t + 1.5·2^52) does the same for every |t| < 2^51; its low word is rint(t).)
+template <typename T>
+struct QBias;
+template <>
+struct QBias<float> {
+    static constexpr int value = 0x4B400000;
+};
+template <>
+struct QBias<double> {
+    static constexpr int value = 0;
+};
+__device__ __forceinline__ void quantize_block(const float (&x)[L], float inv, int (&qb)[L], bool &bad) {
+    bool big[4] = {false, false, false, false};  // independent predicate chains
 #pragma unroll
     for (int i = 0; i < L; i++) {
-        t[i] = __fmul_rn(x[i], inv);
-        big |= !(fabsf(t[i]) < 4194304.0f);
+        const float t = __fmul_rn(x[i], inv);
+        qb[i] = __float_as_int(__fadd_rn(t, 12582912.0f));
+        big[i & 3] |= !(fabsf(t) < 4194304.0f);
     }
-    if (!big) {
-#pragma unroll
-        for (int i = 0; i < L; i++) q[i] = __float_as_int(__fadd_rn(t[i], 12582912.0f)) - 0x4B400000;
-    } else {
+    if ((big[0] || big[1]) || (big[2] || big[3])) {
 #pragma unroll
         for (int i = 0; i < L; i++) {
-            bad |= !(fabsf(t[i]) <= 1073741760.0f);
-            q[i] = __float2int_rn(t[i]);
+            const float t = __fmul_rn(x[i], inv);
+            bad |= !(fabsf(t) <= 1073741760.0f);
+            qb[i] = static_cast<int>(static_cast<uint32_t>(__float2int_rn(t)) + 0x4B400000u);
         }
     }
 }
-__device__ __forceinline__ void quantize_block(const double (&x)[L], double inv, int (&q)[L], bool &bad) {
+__device__ __forceinline__ void quantize_block(const double (&x)[L], double inv, int (&qb)[L], bool &bad) {
 #pragma unroll
     for (int i = 0; i < L; i++) {
         const double t = __dmul_rn(x[i], inv);
         bad |= !(fabs(t) <= 1073741823.0);
-        q[i] = static_cast<int>(static_cast<uint32_t>(__double_as_longlong(__dadd_rn(t, 6755399441055744.0))));
+        qb[i] = static_cast<int>(static_cast<uint32_t>(__double_as_longlong(__dadd_rn(t, 6755399441055744.0))));
     }
 }
 __device__ __forceinline__ float dequantize(int q, float s) { return __fmul_rn(__int2float_rn(q), s); }
 __device__ __forceinline__ double dequantize(int q, double s) {
     return __dmul_rn(__int2double_rn(q), s);
+}
+
+// Align a dynamic shared-memory pointer by offsetting the __shared__ array itself (an
+// integer round trip through uintptr_t would lose the address space, and every access
+// through the result would compile to a generic LD.E/ST.E with 64-bit address math).
+template <uint32_t A>
+__device__ __forceinline__ uint8_t *smem_align(uint8_t *raw) {
+    return raw + ((A - (smem_u32(raw) & (A - 1))) & (A - 1));
 }
 
 // ------------------------------------------------------------------ swizzled tile access
@@ -786,8 +804,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
     unsigned *__restrict__ ticket, uint64_t *__restrict__ d_out_bytes, const HdrStatic hs) {
     using LY = CompLayout<T>;
     extern __shared__ uint8_t smem_raw[];
-    uint8_t *inbuf = reinterpret_cast<uint8_t *>(
-        (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint8_t *inbuf = smem_align<1024>(smem_raw);
     uint8_t *ring = inbuf + LY::IN_BYTES;
     __shared__ uint64_t s_full;                    // input buffer
     __shared__ uint64_t s_staged[NQ], s_done[NQ];  // queue slots
@@ -926,7 +943,9 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
             uint32_t sign = 0, or_rest = 0;
 #pragma unroll
             for (int i = L - 1; i >= 0; i--) {
-                const int d = qv[i] - (i ? qv[i - 1] : 0);
+                // biased patterns difference to d_i (mod 2^32; |d_i| < 2^31 by the range check)
+                const int d = static_cast<int>(static_cast<uint32_t>(qv[i]) -
+                                               static_cast<uint32_t>(i ? qv[i - 1] : QBias<T>::value));
                 a[i] = static_cast<uint32_t>(d < 0 ? -d : d);
                 sign = __funnelshift_l(static_cast<uint32_t>(d), sign, 1);  // bit i = d_i < 0
                 if (i) or_rest |= a[i];
@@ -1178,8 +1197,7 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 3 : 2) decompress_kernel(
                                                            T *__restrict__ out, const Geom g,
                                                            int *__restrict__ d_status) {
     extern __shared__ uint8_t smem_raw[];
-    uint8_t *ostage = reinterpret_cast<uint8_t *>(
-        (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint8_t *ostage = smem_align<1024>(smem_raw);
     uint8_t *ring = ostage + Traits<T>::TILE_BYTES;
     __shared__ uint64_t s_bar[2];
     __shared__ uint32_t s_warp[NT / 32];

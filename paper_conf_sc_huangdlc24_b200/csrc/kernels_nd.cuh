@@ -125,7 +125,7 @@ __global__ void __launch_bounds__(NT) compress_nd_kernel(const T *__restrict__ i
                                                          uint64_t *__restrict__ d_out_bytes,
                                                          const HdrStatic hs) {
     extern __shared__ uint8_t stage_raw[];
-    uint8_t *stage = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(stage_raw) + 15) & ~uintptr_t(15));
+    uint8_t *stage = smem_align<16>(stage_raw);
     __shared__ uint32_t s_warp[NT / 32];
     __shared__ uint32_t s_tk;
     __shared__ uint64_t s_excl;
@@ -307,7 +307,7 @@ __global__ void __launch_bounds__(NT) decompress_nd_kernel(const uint8_t *__rest
                                                            T *__restrict__ out, const GeomND g,
                                                            int *__restrict__ d_status) {
     extern __shared__ uint8_t stage_raw[];
-    uint8_t *pbuf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(stage_raw) + 15) & ~uintptr_t(15));
+    uint8_t *pbuf = smem_align<16>(stage_raw);
     __shared__ uint64_t s_bar;
     __shared__ uint32_t s_warp[NT / 32];
     __shared__ uint64_t s_excl;
