@@ -306,9 +306,11 @@ __device__ __forceinline__ int plane_log2(int fl) { return fl <= 1 ? 0 : 32 - __
 // outlier bytes, then planes A[0..fl). Let ps = st + 4 + nob (plane region), r = ps & 3
 // and P_k the 4 payload bytes at ps + 4k (P_-1, P_-2: header bytes before ps). Every
 // aligned word at ps - r + 4k is funnel(P_k-1, P_k, 8r); those wholly inside the block
-// (k = 0..fl-1, and k = -1 when nob >= r) are plain 32-bit stores, and only the <= 4
-// head and <= 3 tail bytes that share a word with a neighbouring block are written as
-// bytes. SIMT-uniform: no data-dependent branches.
+// (k = 0..fl-1, and k = -1 when nob >= r) are plain 32-bit stores. The <= 4 head and
+// <= 3 tail bytes share an aligned word with a neighbouring block: the staging area is
+// kept zeroed outside live payloads (the resolver clears what it has copied out), so
+// each of the two partial words is merged with a single shared-memory atomicOr.
+// SIMT-uniform: no data-dependent branches.
 template <int R>
 __device__ __forceinline__ void stage_payload(uint8_t *base, uint32_t st, uint32_t sign,
                                               uint32_t outl, int nob, int fl,
@@ -322,10 +324,9 @@ __device__ __forceinline__ void stage_payload(uint8_t *base, uint32_t st, uint32
     uint32_t *w = reinterpret_cast<uint32_t *>(base + ps - r);                   // word k at w[k]
     const bool wm1 = static_cast<uint32_t>(nob) >= r;
     if (wm1) w[-1] = __funnelshift_l(pm2, pm1, sh);
-    const uint32_t head = (ps - r - (wm1 ? 4u : 0u)) - st;                         // 0..4 bytes
-#pragma unroll
-    for (uint32_t j = 0; j < 4; j++)
-        if (j < head) base[st + j] = static_cast<uint8_t>(hdr >> (8 * j));
+    const uint32_t hw = ps - r - (wm1 ? 4u : 0u);  // aligned end of the head bytes
+    const uint32_t head = hw - st;                 // 0..4 bytes: the top bytes of word hw - 4
+    if (head) atomicOr(reinterpret_cast<unsigned *>(base + hw - 4), static_cast<uint32_t>(hdr) << (32 - 8 * head));
     uint32_t prev = pm1, top = pm1;
 #pragma unroll
     for (int k = 0; k < R; k++) {
@@ -335,10 +336,8 @@ __device__ __forceinline__ void stage_payload(uint8_t *base, uint32_t st, uint32
         }
         top = opaque_select(k < fl, A[k], top);
     }
-    const uint32_t e = ps + 4u * fl;  // end of the payload
-#pragma unroll
-    for (uint32_t j = 0; j < 3; j++)
-        if (j < r) base[e - r + j] = static_cast<uint8_t>(top >> (32 - sh + 8 * j));
+    const uint32_t e = ps + 4u * fl;  // end of the payload; its last r bytes are the low bytes of word e - r
+    if (r) atomicOr(reinterpret_cast<unsigned *>(base + e - r), top >> (32 - sh));
 }
 
 // Planes 0..fl-1 of one block from smem at byte position `pos` (any alignment) into
@@ -748,7 +747,7 @@ constexpr uint32_t BAR_PROD = 1;
 template <typename T>
 struct CompLayout {
     static constexpr uint32_t IN_BYTES = Traits<T>::TILE_BYTES;  // one TMA tile
-    static constexpr uint32_t RING = 33792;                      // > one max payload
+    static constexpr uint32_t RING = 32768;  // = the largest tile payload (256 x 128 B); a power of 2
     static constexpr int SMEM = IN_BYTES + RING + 64 + 1024;
 };
 template <typename T>
@@ -856,6 +855,8 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
         }
     };
 
+    for (uint32_t c = tid; c < LY::RING / 16; c += NT_COMP)  // staging ring starts zeroed
+        reinterpret_cast<uint4 *>(ring)[c] = make_uint4(0, 0, 0, 0);
     if (tid == 0) {
         s_end = 0xFFFFFFFFu;
         s_tail = 0;
@@ -1088,9 +1089,15 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
                     if (d_out_bytes) *d_out_bytes = total;
                 }
             }
-            __syncwarp();  // every lane is done reading these ring bytes
+            __syncwarp();  // every lane is done reading these ring bytes: clear them for reuse
+            {
+                uint4 *z = reinterpret_cast<uint4 *>(ring + (pos % LY::RING));
+                for (uint32_t c = lane; c < (agg + 15u) / 16u; c += 32) z[c] = make_uint4(0, 0, 0, 0);
+            }
+            __syncwarp();
             if (lane == 0) {
-                s_tail = pos + agg;  // in order, so the ring frees in order
+                __threadfence_block();  // the zeros land before the producers may reuse the bytes
+                s_tail = pos + agg;     // in order, so the ring frees in order
                 mbar_arrive(&s_done[q]);
             }
         }
