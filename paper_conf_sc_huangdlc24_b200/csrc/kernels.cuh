@@ -143,6 +143,19 @@ __device__ __forceinline__ void quantize_block(const float (&x)[L], float inv, i
         }
     }
 }
+// The same biased patterns with no range check at all. They are exact whenever the
+// block's differences (taken from these patterns, q_{-1} = QBIAS) all satisfy
+// |d_i| < 2^17: then every |qb_i - QBIAS| <= 32 (2^17 - 1) < 2^22, so each
+// s_i = fl(t_i + 1.5·2^23) has its bit pattern strictly inside (2^23, 2^24) — which
+// rounding can only produce from t_i + 1.5·2^23 in [2^23, 2^24), where the RN addition
+// is rint(t_i) exactly and |t_i| < 2^22 passes the range check (NaN and ±Inf have
+// patterns outside that interval). The caller redoes a block with fl_p > 17 through
+// quantize_block().
+constexpr int FAST_FL_MAX = 17;
+__device__ __forceinline__ void quantize_block_unchecked(const float (&x)[L], float inv, int (&qb)[L]) {
+#pragma unroll
+    for (int i = 0; i < L; i++) qb[i] = __float_as_int(__fadd_rn(__fmul_rn(x[i], inv), 12582912.0f));
+}
 __device__ __forceinline__ void quantize_block(const double (&x)[L], double inv, int (&qb)[L], bool &bad) {
 #pragma unroll
     for (int i = 0; i < L; i++) {
@@ -398,6 +411,37 @@ __device__ __forceinline__ uint32_t cta_exclusive_scan(uint32_t v, uint32_t *s_w
     const uint32_t before = __shfl_sync(0xffffffffu, wt, (warp + NW - 1) % NW);
     *total = __shfl_sync(0xffffffffu, wt, NW - 1);
     group_sync(bar_id);
+    return (warp ? before : 0u) + inc - v;
+}
+
+// The compressor's intra-tile scan with ONE barrier: the warp totals (bit 31: some
+// block of the warp was flagged `bad`; a warp's payload total is < 2^31) go to
+// s_warp, which the caller double-buffers by tile parity — a warp can only rewrite
+// a buffer after the next tile's barrier, which every warp reaches only after reading
+// this tile's totals. Also returns the OR of `bad` over the tile.
+__device__ __forceinline__ uint32_t tile_scan_1bar(uint32_t v, bool bad, uint32_t *s_warp,
+                                                   uint32_t *total, bool *any_bad, uint32_t bar_id) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    uint32_t inc = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
+    }
+    const bool wbad = __any_sync(0xffffffffu, bad);
+    if (lane == 31) s_warp[warp] = inc | (wbad ? 0x80000000u : 0u);
+    named_sync(bar_id, NT);
+    constexpr int NW = NT / 32;
+    const uint32_t raw = lane < NW ? s_warp[lane] : 0u;
+    *any_bad = __any_sync(0xffffffffu, (raw >> 31) != 0u);
+    uint32_t wt = raw & 0x7FFFFFFFu;
+#pragma unroll
+    for (int o = 1; o < NW; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, wt, o);
+        if (lane >= o) wt += y;
+    }
+    const uint32_t before = __shfl_sync(0xffffffffu, wt, (warp + NW - 1) % NW);
+    *total = __shfl_sync(0xffffffffu, wt, NW - 1);
     return (warp ? before : 0u) + inc - v;
 }
 
@@ -810,7 +854,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
     __shared__ uint64_t s_qt[NQ];
     __shared__ uint32_t s_qagg[NQ], s_qpos[NQ];
     __shared__ uint8_t s_qbad[NQ];
-    __shared__ uint32_t s_warp[NT / 32];
+    __shared__ uint32_t s_warp[2][NT / 32];  // tile_scan_1bar, by tile parity
     __shared__ uint32_t s_tkin;
     __shared__ uint64_t s_rel;            // producer warps done reading the input buffer
     __shared__ volatile uint32_t s_tail;  // ring bytes released by the resolver
@@ -863,7 +907,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
         mbar_init(&s_rel, NT / 32);
         mbar_init(&s_full, 1);
         for (int i = 0; i < NQ; i++) {
-            mbar_init(&s_staged[i], 1);
+            mbar_init(&s_staged[i], NT / 32);
             mbar_init(&s_done[i], 1);
         }
         fence_mbar_init();
@@ -889,10 +933,10 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
             }
             mbar_wait(&s_full, it & 1);
             const uint64_t t = s_tkin;  // published before the arrival we just waited for
-            if (t >= T_eff) {           // end marker for the resolver
-                if (tid == 0) {
+            if (t >= T_eff) {           // end marker for the resolver (one arrival per warp)
+                if ((tid & 31) == 0) {
                     if (it >= NQ) mbar_wait(&s_done[q], (it / NQ - 1) & 1);
-                    s_end = it;
+                    if (tid == 0) s_end = it;
                     mbar_arrive(&s_staged[q]);
                 }
                 break;
@@ -934,22 +978,42 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
             // ❶ pre-quantization + in-block first-order difference
             bool bad = false;
             int qv[L];
-            quantize_block(x, K.inv, qv, bad);
-            if (!full) {  // tail block: q_i = q_{i-1} past n (FORMAT.md §6.4)
-#pragma unroll
-                for (int i = 1; i < L; i++)
-                    if (i >= (int)valid) qv[i] = qv[i - 1];
-            }
             uint32_t a[L];
             uint32_t sign = 0, or_rest = 0;
+            auto difference = [&]() {
+                if (!full) {  // tail block: q_i = q_{i-1} past n (FORMAT.md §6.4)
 #pragma unroll
-            for (int i = L - 1; i >= 0; i--) {
-                // biased patterns difference to d_i (mod 2^32; |d_i| < 2^31 by the range check)
-                const int d = static_cast<int>(static_cast<uint32_t>(qv[i]) -
-                                               static_cast<uint32_t>(i ? qv[i - 1] : QBias<T>::value));
-                a[i] = static_cast<uint32_t>(d < 0 ? -d : d);
-                sign = __funnelshift_l(static_cast<uint32_t>(d), sign, 1);  // bit i = d_i < 0
-                if (i) or_rest |= a[i];
+                    for (int i = 1; i < L; i++)
+                        if (i >= (int)valid) qv[i] = qv[i - 1];
+                }
+                sign = 0;
+                or_rest = 0;
+#pragma unroll
+                for (int i = L - 1; i >= 0; i--) {
+                    // biased patterns difference to d_i (mod 2^32; |d_i| < 2^31 by the range check)
+                    const int d = static_cast<int>(static_cast<uint32_t>(qv[i]) -
+                                                   static_cast<uint32_t>(i ? qv[i - 1] : QBias<T>::value));
+                    a[i] = static_cast<uint32_t>(d < 0 ? -d : d);
+                    sign = __funnelshift_l(static_cast<uint32_t>(d), sign, 1);  // bit i = d_i < 0
+                    if (i) or_rest |= a[i];
+                }
+            };
+            if constexpr (sizeof(T) == 4) {
+                // unchecked patterns first; a block they may not cover exactly (fl_p > 17,
+                // see quantize_block_unchecked) is redone with the checked quantizer
+                quantize_block_unchecked(x, K.inv, qv);
+                difference();
+                if (32 - __clz(or_rest | a[0]) > FAST_FL_MAX) {
+                    // rare: re-read the block from global memory (x is dead by now, and
+                    // keeping it live would cost registers on the common path)
+#pragma unroll
+                    for (int i = 0; i < L; i++) x[i] = (i < (int)valid) ? in[b * L + i] : T(0);
+                    quantize_block(x, K.inv, qv, bad);
+                    difference();
+                }
+            } else {
+                quantize_block(x, K.inv, qv, bad);
+                difference();
             }
 
             // ❷ fixed lengths and the fine-tuned Plain/Outlier selection
@@ -974,10 +1038,10 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
             }
             if (!K.ok) bad = true;
 
-            const bool any_bad = named_sync_or(BAR_PROD, NT, bad);
-            // intra-tile scan ("Reduce")
+            // intra-tile scan ("Reduce") and the tile's range flag, one barrier
             uint32_t agg;
-            const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg, BAR_PROD);
+            bool any_bad;
+            const uint32_t my_excl = tile_scan_1bar(size, bad, s_warp[it & 1], &agg, &any_bad, BAR_PROD);
             if (tid == 0 && g.T) publish_aggregate(index, t, agg, any_bad);
             if (tid == 0) TRACE(t, 2, gtimer());
             // ring space (16-aligned, contiguous), computed identically by every producer
@@ -1022,19 +1086,25 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
                     }
                 }
             }
-            named_sync(BAR_PROD, NT);  // staging complete
-            if (tid == 0) {
-                TRACE(t, 4, gtimer());
+            // this warp's blocks are staged: one arrival per warp on the queue slot (no
+            // CTA barrier — a warp with nothing to stage goes on to the next tile);
+            // thread 0 fills in the slot first. Every arriving warp waits for the slot
+            // to be free, so s_staged[q] never runs a phase ahead of the resolver.
+            __syncwarp();
+            if ((tid & 31) == 0) {
                 if (it >= NQ) mbar_wait(&s_done[q], (it / NQ - 1) & 1);  // queue slot free
-                s_qt[q] = t;
-                s_qagg[q] = agg;
-                s_qbad[q] = any_bad;
-                s_qpos[q] = pos;
-                mbar_arrive(&s_staged[q]);
-                if (!ahead) {  // claim now, nothing unpublished held: wait for ring room first
-                    while (head - s_tail + 2 * last_agg + 64 > LY::RING && head != s_tail) __nanosleep(64);
-                    claim(atomicAdd(ticket, 1u));
+                if (tid == 0) {
+                    TRACE(t, 4, gtimer());
+                    s_qt[q] = t;
+                    s_qagg[q] = agg;
+                    s_qbad[q] = any_bad;
+                    s_qpos[q] = pos;
                 }
+                mbar_arrive(&s_staged[q]);
+            }
+            if (tid == 0 && !ahead) {  // claim now, nothing unpublished held: wait for ring room first
+                while (head - s_tail + 2 * last_agg + 64 > LY::RING && head != s_tail) __nanosleep(64);
+                claim(atomicAdd(ticket, 1u));
             }
         }
     } else {
@@ -1332,13 +1402,14 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 3 : 2) decompress_kernel(
         const uint32_t fl = obyte & 31u;
         const bool is_o = (obyte & 0x80u) != 0;
         const uint32_t nob = is_o ? ((obyte >> 5) & 3u) + 1u : 0u;
-        bool bad = (!is_o && (obyte & 0x60u));
+        const bool bad = (!is_o && (obyte & 0x60u));
         const uint32_t size = is_o ? 4u + nob + 4u * fl : (fl ? 4u * (1u + fl) : 0u);
+        // one-barrier scan (+ OR of bad): s_warp is next rewritten after the two CTA
+        // barriers below, so it needs no second barrier and no double buffer
         uint32_t agg;
-        const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg);
-        const uint32_t bytes = s_bytes[cur];
-        bad |= (tid == 0 && agg != bytes);
-        if (__syncthreads_or(bad)) {
+        bool any_bad;
+        const uint32_t my_excl = tile_scan_1bar(size, bad, s_warp, &agg, &any_bad, 0);
+        if (any_bad || agg != s_bytes[cur]) {
             err = ST_FORMAT;
             if (tid == 0) {
                 mbar_wait(&s_bar[cur], (it >> 1) & 1);

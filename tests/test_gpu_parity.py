@@ -110,6 +110,28 @@ def test_special_fields(enc):
     check_roundtrip(xh, 1e-3, "abs", enc)
 
 
+@pytest.mark.parametrize("enc", ["plain", "outlier"])
+def test_unchecked_quantizer_boundary(enc):
+    """f32 blocks whose differences sit at the unchecked quantizer's cut-off (fl_p 17 vs
+    18, i.e. |q| up to 32 (2^17 - 1) = 2^22 - 32 on the fast side) and ties near 2^21:
+    both sides of the cut must give the oracle's bytes (kernels.cuh FAST_FL_MAX)."""
+    rng = np.random.default_rng(2024)
+    nblk = 600
+    lim = np.array([2**16, 2**17 - 1, 2**17, 2**17 + 1, 2**18])[rng.integers(0, 5, nblk)]
+    steps = rng.integers(-1, 2, (nblk, 32)) * lim[:, None]          # steps of 0, ±lim
+    steps[::7] = np.abs(steps[::7])                                   # monotone ramps to ~2^22
+    steps[::11] = lim[::11, None]                                     # exactly 32 lim
+    q = np.cumsum(steps, axis=1).reshape(-1).astype(np.float64)
+    xh = q.astype(np.float32)
+    xh[::13] += 0.5                                                   # ties, even and odd
+    check_roundtrip(xh, 0.5, "abs", enc)
+    near = (2.0**21 + np.arange(-4000, 4000) + 0.5).astype(np.float32)  # ties near 2^21
+    check_roundtrip(near, 0.5, "abs", enc)
+    big = np.float32(2.0**22) + np.arange(-3000, 3000).astype(np.float32)  # |q| around 2^22
+    check_roundtrip(big, 0.5, "abs", enc)
+    check_roundtrip(-big, 0.5, "abs", enc)
+
+
 def test_range_status_header_parity():
     xh = np.linspace(0, 1, 10000).astype(np.float32)
     xh[5000] = 3e9
