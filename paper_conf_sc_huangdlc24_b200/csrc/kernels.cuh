@@ -265,7 +265,8 @@ __device__ __forceinline__ void swap_stage(uint32_t (&A)[32]) {
 template <int S>
 __device__ __forceinline__ void merge_stage(uint32_t (&A)[32]) {
 #pragma unroll
-    for (int i = 0; i < S; i++) A[i] |= A[i + S] << S;
+    // the bits are disjoint, so + is |: one IMAD or LEA per row instead of SHL + LOP3
+    for (int i = 0; i < S; i++) A[i] = A[i + S] * (1u << S) + A[i];
 }
 template <int S>
 __device__ __forceinline__ void split_stage(uint32_t (&A)[32]) {
@@ -1186,42 +1187,44 @@ __device__ __forceinline__ void decode_block(const uint8_t *pbuf, uint32_t pos, 
     const bool is_o = (obyte & 0x80u) != 0;
     const uint32_t nob = is_o ? ((obyte >> 5) & 3u) + 1u : 0u;
     uint32_t a[L];
-#pragma unroll
-    for (int i = 0; i < L; i++) a[i] = 0;
-    uint32_t sign = 0;
+    uint32_t sign = 0, outlier = 0;
     const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, size ? fl : 0u));
     if (size) {
         sign = ld_u32_unaligned(pbuf, pos);
         pos += 4;
-        uint32_t outlier = 0;
         if (is_o) {
             outlier = ld_u32_unaligned(pbuf, pos);
             if (nob < 4) outlier &= (1u << (8 * nob)) - 1u;
             pos += nob;
         }
-        if (flw > 0) {
-            if (flw <= 1) {
-                load_planes<1>(pbuf, pos, fl, a);
-                unpack_planes<0>(a);
-            } else if (flw <= 2) {
-                load_planes<2>(pbuf, pos, fl, a);
-                unpack_planes<1>(a);
-            } else if (flw <= 4) {
-                load_planes<4>(pbuf, pos, fl, a);
-                unpack_planes<2>(a);
-            } else if (flw <= 8) {
-                load_planes<8>(pbuf, pos, fl, a);
-                unpack_planes<3>(a);
-            } else if (flw <= 16) {
-                load_planes<16>(pbuf, pos, fl, a);
-                unpack_planes<4>(a);
-            } else {
-                load_planes<32>(pbuf, pos, fl, a);
-                unpack_planes<5>(a);
-            }
-        }
-        if (is_o) a[0] = outlier;
     }
+    // every row of a[] is written once: zeros, or load_planes (rows < R; a block with
+    // size 0 has fl 0, so its planes load as zeros) + unpack_planes (rows >= R)
+    if (flw == 0) {
+#pragma unroll
+        for (int i = 0; i < L; i++) a[i] = 0;
+    } else {
+        if (flw <= 1) {
+            load_planes<1>(pbuf, pos, fl, a);
+            unpack_planes<0>(a);
+        } else if (flw <= 2) {
+            load_planes<2>(pbuf, pos, fl, a);
+            unpack_planes<1>(a);
+        } else if (flw <= 4) {
+            load_planes<4>(pbuf, pos, fl, a);
+            unpack_planes<2>(a);
+        } else if (flw <= 8) {
+            load_planes<8>(pbuf, pos, fl, a);
+            unpack_planes<3>(a);
+        } else if (flw <= 16) {
+            load_planes<16>(pbuf, pos, fl, a);
+            unpack_planes<4>(a);
+        } else {
+            load_planes<32>(pbuf, pos, fl, a);
+            unpack_planes<5>(a);
+        }
+    }
+    if (is_o) a[0] = outlier;
     int qv = 0;
 #pragma unroll
     for (int i = 0; i < L; i++) {
