@@ -52,6 +52,9 @@ def parse():
     ap.add_argument("--cpu-sample-log2", type=int, default=28,
                     help="values in the oracle cpu_baseline sample (2^k)")
     ap.add_argument("--no-plain", action="store_true", help="skip the secondary Plain-mode pass")
+    ap.add_argument("--rel-scope", default="rank", choices=["rank", "global"],
+                    help="REL range per rank's slab (default; no extra collective) or of the whole "
+                         "field (one 16-byte NCCL all-reduce of (min, -max); SURVEY 8(e))")
     return ap.parse_args()
 
 
@@ -62,14 +65,6 @@ def dist_env():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     return rank, world, local
-
-
-def slab(n: int, world: int, rank: int):
-    """Block-aligned contiguous slab of rank r."""
-    S = -(-n // world)
-    S = -(-S // 32) * 32
-    s0 = min(n, rank * S)
-    return s0, min(n, s0 + S) - s0
 
 
 def load_peaks():
@@ -207,6 +202,7 @@ def main():
         return run_reference(args)
 
     import paper_conf_sc_huangdlc24_b200 as cz
+    from paper_conf_sc_huangdlc24_b200.multi import reduce_range, slab
 
     rank, world, local = dist_env()
     if world != args.gpus and world > 1:
@@ -235,10 +231,17 @@ def main():
     offsets = torch.zeros(world + 1, dtype=torch.int64, device=dev)
     stream = torch.cuda.current_stream(dev)
 
+    glob = args.rel_scope == "global" and spec.eb_mode == "rel"
+    rng_work = torch.empty(8, dtype=torch.float64, device=dev)
+
     def step(evs=None, enc=args.enc):
         if evs:
             evs[0].record(stream)
-        cz.compress_prepare(x, lam, spec.eb_mode, out, stream=stream)
+        if glob:  # value range -> 16-byte all-reduce -> eb_abs from the global range
+            cz.value_range(x, work=rng_work, stream=stream)
+            cz.compress_prepare_range(x, lam, reduce_range(rng_work), out, stream=stream)
+        else:
+            cz.compress_prepare(x, lam, spec.eb_mode, out, stream=stream)
         if evs:
             evs[1].record(stream)
         cz.compress_encode(x, lam, spec.eb_mode, enc, out, nbytes, stream=stream)
@@ -353,9 +356,10 @@ def main():
         torch.cuda.synchronize()
 
     # cpu_baseline: the oracle as it stands, on a bounded sample, rank 0 at N=1 only
-    cpu = None
+    cpu = cpu_mt = None
     if rank == 0 and world == 1:
         cpu = run_cpu_baseline(args, x, lam, spec)
+        cpu_mt = run_cpu_baseline_all_cores(args, x, lam, spec)
 
     # e2e through the host-buffer C-ABI calls (pinned host memory, copies timed)
     e2e = run_e2e(args, cz, x, y, out, dev, stream, lam, spec, dist, world, n_total, w)
@@ -372,7 +376,9 @@ def main():
                        "n_values": n_total, "values_per_rank": cnt, "eb_mode": spec.eb_mode,
                        "eb": lam, "enc_mode": args.enc,
                        "l2": "inputs larger than L2 (field >> 126 MB); no flush needed",
-                       "parallelism": f"slab x{world}, NCCL all-gather of compressed sizes"},
+                       "rel_scope": args.rel_scope,
+                       "parallelism": f"slab x{world}, NCCL all-gather of compressed sizes"
+                                      + (" + all-reduce of the value range" if glob else "")},
             "comp_gbs": round(comp_gbs, 1), "decomp_gbs": round(decomp_gbs, 1),
             "cr": round(n_total * w / stream_total, 3), "psnr_db": round(psnr, 3),
             "eb_abs_rank0": hdr["eb_abs"],
@@ -380,6 +386,7 @@ def main():
                          "allgather_index": round(gather_ms, 4), "decompress_kernel": round(dec_ms, 4)},
             "roofline": roof,
             "cpu_baseline": cpu,
+            "cpu_baseline_all_cores": cpu_mt,
             "e2e": e2e,
             "clocks": clocks,
             "gpu_launches": args.steps * (3 + (1 if world > 1 else 0)),
@@ -461,6 +468,38 @@ def run_cpu_baseline(args, x, lam, spec):
             "seconds": round(t2 - t0, 2),
             "sample": f"first {m} values ({xs.nbytes / 2**30:.2f} GiB) of the rank-0 slab, one "
                       f"compress + decompress, single-threaded C oracle (REL range of the sample)"}
+
+
+def run_cpu_baseline_all_cores(args, x, lam, spec):
+    """SURVEY §8(d)'s second CPU baseline: the same oracle over block-aligned chunks of
+    the same sample on every host core (ctypes releases the GIL; one thread per core):
+    the REL range of the sample (one oracle pass), then per-chunk compress and
+    decompress in parallel. Chunk streams are separate (no serial concatenation)."""
+    import concurrent.futures as cf
+
+    import oracle
+
+    m = min(x.numel(), 1 << args.cpu_sample_log2)
+    xs = x[:m].cpu().numpy()
+    cores = os.cpu_count() or 1
+    enc = oracle.OUTLIER if args.enc == "outlier" else oracle.PLAIN
+    ebm = oracle.REL if spec.eb_mode == "rel" else oracle.ABS
+    step = -(-m // cores)
+    step = -(-step // 8192) * 8192
+    chunks = [xs[i:i + step] for i in range(0, m, step)]
+    with cf.ThreadPoolExecutor(max_workers=cores) as ex:
+        t0 = time.perf_counter()
+        eb_abs = oracle.resolve_eb(xs, lam, ebm)
+        streams = list(ex.map(lambda c: oracle.compress(c, eb_abs, oracle.ABS, enc)[0], chunks))
+        t1 = time.perf_counter()
+        list(ex.map(lambda a: oracle.decompress(a[0], a[1].size, a[1].dtype), zip(streams, chunks)))
+        t2 = time.perf_counter()
+    gb = xs.nbytes / 1e9
+    return {"value": round(gb / (t2 - t0), 4), "unit": "GB/s", "cores": min(cores, len(chunks)),
+            "kind": "oracle", "comp_gbs": round(gb / (t1 - t0), 4), "decomp_gbs": round(gb / (t2 - t1), 4),
+            "seconds": round(t2 - t0, 2),
+            "sample": f"the cpu_baseline sample in {len(chunks)} block-aligned chunks, one oracle "
+                      f"thread per core (REL range by one serial oracle pass)"}
 
 
 if __name__ == "__main__":

@@ -90,6 +90,24 @@ int cszp2_compress_prepare(const void *d_in, uint64_t n, int dtype, double eb, i
 int cszp2_compress_encode(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
                           int enc_mode, void *d_out, uint64_t *d_out_bytes, void *stream);
 
+/* Global REL for one field sharded across ranks (the paper's REL bound
+ * is relative to the value range of the whole dataset). Per rank:
+ *   cszp2_value_range(slab) -> reduce (min, max) across ranks (the caller's one
+ *   16-byte collective) -> cszp2_compress_prepare_range(slab, lambda, range)
+ *   -> cszp2_compress_encode(slab, lambda, CSZP2_EB_REL, ...).
+ * The ranks' offset bytes and payloads then concatenate to the single-GPU stream's.
+ * cszp2_value_range: d_work = 8 doubles (64 B, 16-byte aligned, device); on
+ *   completion (stream-ordered) d_work[0] = min, d_work[1] = max over the non-NaN
+ *   values of d_in, exact (T -> f64 conversions); (+inf, -inf) when there is none
+ *   (n = 0 or all NaN). The other words are scratch. Errors: ARG, CUDA.
+ * cszp2_compress_prepare_range: as cszp2_compress_prepare with eb_mode REL, except
+ *   that eb_abs = eb * (max - min) comes from the device range d_range[0..1]
+ *   (16-byte aligned) instead of a reduction over d_in; a zero or empty range gives
+ *   eb_abs = eb, as for the local range (FORMAT.md §6.1). Errors as prepare. */
+int cszp2_value_range(const void *d_in, uint64_t n, int dtype, double *d_work, void *stream);
+int cszp2_compress_prepare_range(const void *d_in, uint64_t n, int dtype, double eb,
+                                 const double *d_range, void *d_out, void *stream);
+
 /* cszp2_compress_encode with ablation flags (NEXT #2; same stream bytes either way):
  *  CSZP2_FLAG_CHAINED_SCAN: replace the decoupled lookback by the plain chained
  *    scan it improves on (Fig 12 left; the Fig 17 comparison).

@@ -63,6 +63,8 @@ def _load():
     L.cszp2_compress.argtypes = sig
     L.cszp2_compress_encode.argtypes = sig
     L.cszp2_compress_prepare.argtypes = [vp, u64, i32, dbl, i32, vp, vp]
+    L.cszp2_value_range.argtypes = [vp, u64, i32, vp, vp]
+    L.cszp2_compress_prepare_range.argtypes = [vp, u64, i32, dbl, vp, vp, vp]
     L.cszp2_compress_encode_ex.argtypes = [vp, u64, i32, dbl, i32, i32, vp, vp, ctypes.c_uint, vp]
     L.cszp2_decompress.argtypes = [vp, vp, u64, i32, vp, vp]
     L.cszp2_read_header.argtypes = [vp, ctypes.POINTER(Header), vp]
@@ -86,7 +88,7 @@ _lib = _load()
 LIBRARY_PATH = _LIB_PATH
 EXPORTED = (
     "cszp2_compress_bound", "cszp2_compress", "cszp2_compress_prepare", "cszp2_compress_encode",
-    "cszp2_compress_encode_ex",
+    "cszp2_compress_encode_ex", "cszp2_value_range", "cszp2_compress_prepare_range",
     "cszp2_decompress", "cszp2_decompress_range", "cszp2_read_header", "cszp2_compress_host", "cszp2_decompress_host",
     "cszp2_container_index", "cszp2_version",
     "cszp2_compress_bound_nd", "cszp2_compress_nd", "cszp2_decompress_nd",
@@ -153,6 +155,30 @@ def compress_encode(x, eb, eb_mode, enc_mode, out, out_bytes=None, stream=None):
     rc = _lib.cszp2_compress_encode(_ptr(x), x.numel(), _DT[x.dtype], float(eb), _EB[eb_mode],
                                     _ENC[enc_mode], _ptr(out), _ptr(out_bytes), _stream(stream))
     _check("cszp2_compress_encode", rc)
+
+
+def value_range(x: torch.Tensor, work=None, stream=None) -> torch.Tensor:
+    """Device (min, max) of the non-NaN values of x as float64 (+inf, -inf if none):
+    returns an 8-element float64 work tensor whose first two words hold them."""
+    _need_cuda(x, work)
+    x = x.contiguous().view(-1)
+    if work is None:
+        work = torch.empty(8, dtype=torch.float64, device=x.device)
+    rc = _lib.cszp2_value_range(_ptr(x), x.numel(), _DT[x.dtype], _ptr(work), _stream(stream))
+    _check("cszp2_value_range", rc)
+    return work
+
+
+def compress_prepare_range(x, eb, rng: torch.Tensor, out, stream=None):
+    """compress_prepare for REL with a caller-supplied device range rng[0:2] =
+    (min, max), e.g. reduced across ranks (global REL); then compress_encode(x, eb,
+    "rel", ...)."""
+    _need_cuda(x, rng, out)
+    if rng.dtype != torch.float64 or rng.numel() < 2 or not rng.is_contiguous():
+        raise ValueError("rng must be a contiguous float64 CUDA tensor of >= 2 elements")
+    rc = _lib.cszp2_compress_prepare_range(_ptr(x), x.numel(), _DT[x.dtype], float(eb), _ptr(rng),
+                                           _ptr(out), _stream(stream))
+    _check("cszp2_compress_prepare_range", rc)
 
 
 FLAG_CHAINED_SCAN = 1

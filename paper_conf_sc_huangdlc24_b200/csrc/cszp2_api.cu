@@ -116,7 +116,8 @@ int check_compress_args(const void *d_in, uint64_t n, int dtype, double eb, int 
 }
 
 template <typename T>
-int launch_minmax(const void *d_in, uint64_t n, double lambda, void *d_out, cudaStream_t st) {
+int launch_minmax(const void *d_in, uint64_t n, double lambda, void *d_out, cudaStream_t st,
+                  double *range_out = nullptr) {
     const int sms = sm_count();
     const uint64_t nchunks = n * sizeof(T) / MM_CHUNK;
     if (nchunks >= static_cast<uint64_t>(sms)) {  // bulk-TMA streaming, 2 CTAs per SM
@@ -132,14 +133,14 @@ int launch_minmax(const void *d_in, uint64_t n, double lambda, void *d_out, cuda
         const uint64_t want = 2ull * sms;
         const int grid = static_cast<int>(nchunks < want ? nchunks : want);
         minmax_kernel_tma<T><<<grid, 256, smem, st>>>(static_cast<const T *>(d_in), n, lambda,
-                                                       static_cast<uint8_t *>(d_out));
+                                                       static_cast<uint8_t *>(d_out), range_out);
         return launch_status();
     }
     const uint64_t nvec = n / (16 / sizeof(T));
     uint64_t want = (nvec + 255) / 256;
     int grid = static_cast<int>(want < 1 ? 1 : (want > (uint64_t)sms * 8 ? (uint64_t)sms * 8 : want));
     minmax_kernel<T><<<grid, 256, 0, st>>>(static_cast<const T *>(d_in), n, lambda,
-                                            static_cast<uint8_t *>(d_out));
+                                            static_cast<uint8_t *>(d_out), range_out);
     return launch_status();
 }
 
@@ -303,6 +304,28 @@ int cszp2_compress_prepare(const void *d_in, uint64_t n, int dtype, double eb, i
         return dtype == CSZP2_F32 ? launch_minmax<float>(d_in, n, eb, d_out, S(stream))
                                   : launch_minmax<double>(d_in, n, eb, d_out, S(stream));
     return CSZP2_OK;
+}
+
+int cszp2_value_range(const void *d_in, uint64_t n, int dtype, double *d_work, void *stream) {
+    if (!wsize(dtype) || !d_work || (!d_in && n)) return CSZP2_ERR_ARG;
+    if ((n && !aligned16(d_in)) || !aligned16(d_work) || n > (1ull << 40)) return CSZP2_ERR_ARG;
+    // d_work[0..1]: the result; bytes 32..63: the reduction's header-shaped scratch
+    if (cudaMemsetAsync(d_work, 0, 8 * sizeof(double), S(stream)) != cudaSuccess) return CSZP2_ERR_CUDA;
+    return dtype == CSZP2_F32 ? launch_minmax<float>(d_in, n, 1.0, d_work, S(stream), d_work)
+                              : launch_minmax<double>(d_in, n, 1.0, d_work, S(stream), d_work);
+}
+
+int cszp2_compress_prepare_range(const void *d_in, uint64_t n, int dtype, double eb,
+                                 const double *d_range, void *d_out, void *stream) {
+    int rc = check_compress_args(d_in, n, dtype, eb, CSZP2_EB_REL, d_out);
+    if (rc) return rc;
+    if (!d_range || !aligned16(d_range)) return CSZP2_ERR_ARG;
+    Geom g = geometry(n);
+    if (cudaMemsetAsync(d_out, 0, g.O, S(stream)) != cudaSuccess ||
+        cudaMemsetAsync(static_cast<uint8_t *>(d_out) + stream_bound(g), 0, 16, S(stream)) != cudaSuccess)
+        return CSZP2_ERR_CUDA;
+    eb_from_range_kernel<<<1, 1, 0, S(stream)>>>(d_range, eb, static_cast<uint8_t *>(d_out));
+    return launch_status();
 }
 
 int cszp2_compress_encode_ex(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,

@@ -594,7 +594,8 @@ __device__ __forceinline__ double unsortable(unsigned long long u) {
 // Block reduction of (mn, mx), sortable-integer atomics into the header scratch, and
 // the last CTA's finalisation: eb_abs = λ·(max − min) (R-15). Every thread calls it.
 template <typename T>
-__device__ __forceinline__ void minmax_finish(T mn, T mx, double lambda, uint8_t *__restrict__ hdr) {
+__device__ __forceinline__ void minmax_finish(T mn, T mx, double lambda, uint8_t *__restrict__ hdr,
+                                              double *__restrict__ range_out) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
         mn = fmin(mn, __shfl_xor_sync(0xffffffffu, mn, o));
@@ -631,18 +632,29 @@ __device__ __forceinline__ void minmax_finish(T mn, T mx, double lambda, uint8_t
     __syncthreads();
     if (s_last && threadIdx.x == 0) {
         __threadfence();
-        double r = 0.0;
+        double r = 0.0, dmn = INFINITY, dmx = -INFINITY;  // (+inf, -inf): no non-NaN value
         if (sizeof(T) == 4) {
             unsigned emx = atomicAdd(reinterpret_cast<unsigned *>(hdr + 40), 0u);
             unsigned emn = ~atomicAdd(reinterpret_cast<unsigned *>(hdr + 48), 0u);
-            if (emx != 0u)
-                r = __dsub_rn((double)unsortable(emx), (double)unsortable(emn));
+            if (emx != 0u) {
+                dmn = (double)unsortable(emn);
+                dmx = (double)unsortable(emx);
+                r = __dsub_rn(dmx, dmn);
+            }
         } else {
             unsigned long long emx =
                 atomicAdd(reinterpret_cast<unsigned long long *>(hdr + 40), 0ull);
             unsigned long long emn =
                 ~atomicAdd(reinterpret_cast<unsigned long long *>(hdr + 48), 0ull);
-            if (emx != 0ull) r = __dsub_rn(unsortable(emx), unsortable(emn));
+            if (emx != 0ull) {
+                dmn = unsortable(emn);
+                dmx = unsortable(emx);
+                r = __dsub_rn(dmx, dmn);
+            }
+        }
+        if (range_out) {
+            range_out[0] = dmn;
+            range_out[1] = dmx;
         }
         const double eb_abs = (r == 0.0) ? lambda : __dmul_rn(lambda, r);
         *reinterpret_cast<double *>(hdr + 32) = eb_abs;
@@ -656,7 +668,8 @@ __device__ __forceinline__ void minmax_finish(T mn, T mx, double lambda, uint8_t
 // CTA restores zeros): [40] sortable max, [48] ~sortable min, [56] u32 CTA counter.
 template <typename T>
 __global__ void __launch_bounds__(256) minmax_kernel(const T *__restrict__ in, uint64_t n,
-                                                     double lambda, uint8_t *__restrict__ hdr) {
+                                                     double lambda, uint8_t *__restrict__ hdr,
+                                                     double *__restrict__ range_out) {
     using V = typename std::conditional<sizeof(T) == 4, float4, double2>::type;
     constexpr int PER = 16 / sizeof(T);
     T mn = INFINITY, mx = -INFINITY;
@@ -693,7 +706,7 @@ __global__ void __launch_bounds__(256) minmax_kernel(const T *__restrict__ in, u
         mn = fmin(mn, e);
         mx = fmax(mx, e);
     }
-    minmax_finish<T>(mn, mx, lambda, hdr);
+    minmax_finish<T>(mn, mx, lambda, hdr, range_out);
 }
 
 // The same reduction with the field streamed through shared memory by 1D bulk TMA
@@ -702,11 +715,22 @@ __global__ void __launch_bounds__(256) minmax_kernel(const T *__restrict__ in, u
 // register-staged loop above cannot (it tops out near 6.6 TB/s, this near the HBM read
 // rate). d_in is 16-byte aligned (cszp2_compress contract); the bytes past the last
 // whole chunk are read directly by CTA 0.
+// Global REL: eb_abs = λ·(max − min) from a range the caller reduced
+// across ranks (range[0] = min, range[1] = max as f64; min > max: no value), with the
+// same arithmetic and zero-range rule as minmax_finish.
+__global__ void eb_from_range_kernel(const double *__restrict__ range, double lambda,
+                                     uint8_t *__restrict__ hdr) {
+    const double mn = range[0], mx = range[1];
+    const double r = (mn <= mx) ? __dsub_rn(mx, mn) : 0.0;
+    *reinterpret_cast<double *>(hdr + 32) = (r == 0.0) ? lambda : __dmul_rn(lambda, r);
+}
+
 constexpr uint32_t MM_CHUNK = 16384;
 constexpr int MM_STAGES = 4;
 template <typename T>
 __global__ void __launch_bounds__(256) minmax_kernel_tma(const T *__restrict__ in, uint64_t n,
-                                                         double lambda, uint8_t *__restrict__ hdr) {
+                                                         double lambda, uint8_t *__restrict__ hdr,
+                                                     double *__restrict__ range_out) {
     extern __shared__ __align__(128) uint8_t mm_smem[];
     __shared__ uint64_t s_full[MM_STAGES];
     using V = typename std::conditional<sizeof(T) == 4, float4, double2>::type;
@@ -755,7 +779,7 @@ __global__ void __launch_bounds__(256) minmax_kernel_tma(const T *__restrict__ i
             mx = fmax(mx, in[i]);
         }
     }
-    minmax_finish<T>(mn, mx, lambda, hdr);
+    minmax_finish<T>(mn, mx, lambda, hdr, range_out);
 }
 
 // ------------------------------------------------------------------ compression

@@ -39,13 +39,42 @@ def gather_sizes(nbytes: torch.Tensor, group=None) -> torch.Tensor:
     return out
 
 
-def compress_slab(x_slab: torch.Tensor, eb: float, eb_mode: str, enc_mode: str, out=None,
-                  nbytes=None, group=None, stream=None):
-    """Compress this rank's slab and build the container index on the device:
-    returns (stream buffer, this rank's size tensor, offsets int64[world+1])."""
-    from . import compress, container_index
+def reduce_range(rng: torch.Tensor, group=None) -> torch.Tensor:
+    """Global (min, max) from every rank's (min, max) in rng[0:2] (float64): one
+    16-byte all-reduce of (min, -max) with MIN (optional global REL)."""
+    t = torch.stack([rng[0], -rng[1]])
+    if dist.is_available() and dist.is_initialized():
+        dist.all_reduce(t, op=dist.ReduceOp.MIN, group=group)
+    return torch.stack([t[0], -t[1]]).contiguous()
 
-    out, nbytes = compress(x_slab, eb, eb_mode, enc_mode, out=out, out_bytes=nbytes, stream=stream)
+
+def compress_slab(x_slab: torch.Tensor, eb: float, eb_mode: str, enc_mode: str, out=None,
+                  nbytes=None, group=None, stream=None, rel_scope: str = "rank"):
+    """Compress this rank's slab and build the container index on the device:
+    returns (stream buffer, this rank's size tensor, offsets int64[world+1]).
+
+    rel_scope (REL only): "rank" — each rank's own slab range r_s <= r, which still
+    meets the dataset-level bound (P:231) with no extra collective (the default);
+    "global" — the whole field's range through one 16-byte all-reduce, so that the
+    ranks' offset bytes and payloads concatenate to the single-GPU stream's."""
+    from . import (compress, compress_bound, compress_encode, compress_prepare_range,
+                   container_index, value_range)
+
+    if rel_scope not in ("rank", "global"):
+        raise ValueError("rel_scope must be 'rank' or 'global'")
+    if eb_mode == "rel" and rel_scope == "global":
+        x = x_slab.contiguous().view(-1)
+        if out is None:
+            out = torch.empty(compress_bound(x.numel(), x.dtype), dtype=torch.uint8, device=x.device)
+        if nbytes is None:
+            nbytes = torch.zeros(1, dtype=torch.int64, device=x.device)
+        cur = torch.cuda.current_stream() if stream is None else stream
+        with torch.cuda.stream(cur):  # the collective runs on the stream the kernels use
+            rng = reduce_range(value_range(x, stream=cur), group)
+            compress_prepare_range(x, eb, rng, out, stream=cur)
+            compress_encode(x, eb, "rel", enc_mode, out, nbytes, stream=cur)
+    else:
+        out, nbytes = compress(x_slab, eb, eb_mode, enc_mode, out=out, out_bytes=nbytes, stream=stream)
     if dist.is_available() and dist.is_initialized():
         sizes = gather_sizes(nbytes, group)
     else:

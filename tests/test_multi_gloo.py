@@ -163,3 +163,55 @@ def test_compressed_all_gather_two_ranks(orc, enc):
         assert stats["sizes"] == sizes
         assert stats["slot"] == (max(sizes) + 15) // 16 * 16
         assert stats["wire_bytes"] == world * stats["slot"] < stats["raw_bytes"]
+
+
+def _grel_worker(rank, world, port, n, lam, enc, result_q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        from paper_conf_sc_huangdlc24_b200.multi import reduce_range, slab
+        from synthetic import make_field
+
+        s0, cnt = slab(n, world, rank)
+        x = make_field("cfg2", "cpu", s0, cnt).numpy()
+        local = torch.tensor([np.nanmin(x).astype(np.float64), np.nanmax(x).astype(np.float64)])
+        rng = reduce_range(local)  # the product's 16-byte all-reduce (gloo here, NCCL on GPUs)
+        eb_abs = lam * (float(rng[1]) - float(rng[0]))  # FORMAT.md §6.1 on the global range
+        s, rc = oracle.compress(x, eb_abs, oracle.ABS, enc)
+        result_q.put((rank, rc, rng.tolist(), local.tolist(), eb_abs, s.tobytes()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("enc", [0, 1])
+def test_global_rel_two_ranks_matches_single_stream(orc, enc):
+    """SURVEY §8(e) optional global REL: the reduced range is the field's, so every
+    rank quantizes with the single-GPU eb_abs and the ranks' offset bytes and
+    payloads concatenate to the REL stream of the whole field."""
+    world, n, lam = 2, 5 * 8192 + 32 * 3 + 9, 1e-3
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_grel_worker, args=(r, world, port, n, lam, enc, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted([q.get(timeout=120) for _ in range(world)])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    from synthetic import make_field
+
+    full_x = make_field("cfg2", "cpu", 0, n).numpy()
+    full, rc = orc.compress(full_x, lam, orc.REL, enc)
+    assert rc == orc.OK and all(r[1] == orc.OK for r in res)
+    gmin, gmax = float(np.nanmin(full_x)), float(np.nanmax(full_x))
+    for r in res:
+        assert r[2] == [gmin, gmax]                       # every rank holds the global range
+        assert r[3][0] >= gmin and r[3][1] <= gmax
+    pf = sp.parse(full)
+    assert pf["header"]["eb_abs"] == res[0][4] == res[1][4]
+    parts = [sp.parse(np.frombuffer(r[5], np.uint8)) for r in res]
+    np.testing.assert_array_equal(np.concatenate([p["offsets"] for p in parts]), pf["offsets"])
+    np.testing.assert_array_equal(np.concatenate([p["q"] for p in parts]), pf["q"])
