@@ -86,7 +86,7 @@ class ClockSampler:
     def __init__(self, gpu_index: int):
         self.gpu = gpu_index
         self.proc = None
-        self.lines = []
+        self.raw = []
 
     def __enter__(self):
         try:
@@ -95,22 +95,35 @@ class ClockSampler:
                  "-lms", "50"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
+            # nvidia-smi takes a few hundred ms to start: wait for its first sample, so
+            # the timed region (often < 1 s) is covered, and keep only samples taken
+            # between entry and exit
+            deadline = time.monotonic() + 5.0
+            while not self.raw and time.monotonic() < deadline and self.proc.poll() is None:
+                time.sleep(0.01)
         except Exception:
             self.proc = None
+        self.t_in = time.monotonic()
         return self
 
     def _read(self):
         for line in self.proc.stdout:
-            self.lines.append(line.strip())
+            self.raw.append((time.monotonic(), line.strip()))
 
     def __exit__(self, *a):
+        self.t_out = time.monotonic()
         if self.proc:
-            time.sleep(0.15)
+            time.sleep(0.06)  # the sample in flight at exit still belongs to the region
             self.proc.terminate()
             try:
                 self.proc.wait(timeout=2)
             except Exception:
                 self.proc.kill()
+
+    @property
+    def lines(self):
+        t_out = getattr(self, "t_out", float("inf")) + 0.06
+        return [l for t, l in self.raw if self.t_in <= t <= t_out]
 
     def summary(self):
         sm, mx, reasons = [], None, set()
