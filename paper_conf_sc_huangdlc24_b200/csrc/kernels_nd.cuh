@@ -303,7 +303,7 @@ __global__ void __launch_bounds__(NT) compress_nd_kernel(const T *__restrict__ i
 }
 
 template <typename T, int NDIM>
-__global__ void __launch_bounds__(NT) decompress_nd_kernel(const uint8_t *__restrict__ cmp,
+__global__ void __launch_bounds__(NT, 3) decompress_nd_kernel(const uint8_t *__restrict__ cmp,
                                                            T *__restrict__ out, const GeomND g,
                                                            int *__restrict__ d_status) {
     extern __shared__ uint8_t stage_raw[];
