@@ -233,12 +233,8 @@ __global__ void __launch_bounds__(NT) compress_nd_kernel(const T *__restrict__ i
     //      values 0..31 then 32..63), bit planes by two in-register transposes
     const uint32_t outl = a[0];
     if (OUTLIER && nob) a[0] = 0;
-    uint32_t lo[32], hi[32];
-#pragma unroll
-    for (int i = 0; i < 32; i++) {
-        lo[i] = a[i];
-        hi[i] = a[32 + i];
-    }
+    uint32_t(&lo)[32] = *reinterpret_cast<uint32_t(*)[32]>(&a[0]);   // values 0..31
+    uint32_t(&hi)[32] = *reinterpret_cast<uint32_t(*)[32]>(&a[32]);  // values 32..63
     const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, static_cast<unsigned>(size ? fl : 0)));
     if (flw > 0) {
         if (flw <= 4) {

@@ -354,3 +354,30 @@ def test_decompress_tilewise_ablation(n, dtype, locate):
     assert int(st.item()) == 0
     iv = np.uint32 if dtype == np.float32 else np.uint64
     np.testing.assert_array_equal(y.cpu().numpy().view(iv), yr.view(iv))
+
+
+@pytest.mark.parametrize("seed", range(24))
+def test_randomized_parity(seed):
+    """Seeded random mixtures (smooth + noise + spikes + ±0 / denormals / huge values,
+    random n, eb mode, bound and encoding): whole-stream bytes and decompressed bits
+    equal the oracle's. Covers both sides of the unchecked-quantizer cut (fl_p 17/18)
+    and of the F2I fallback (|t| >= 2^22) inside one field."""
+    rng = np.random.default_rng(1000 + seed)
+    dtype = np.float32 if seed % 3 else np.float64
+    n = int(rng.integers(1, 5 * 8192 + 97))
+    i = np.arange(n)
+    base = np.sin(i / rng.uniform(5, 500)) * rng.uniform(0.1, 1e4)
+    noise = rng.standard_normal(n) * rng.choice([0.0, 1e-3, 1.0, 1e2])
+    x = base + noise
+    eb_mode = "rel" if seed % 2 else "abs"
+    eb = float(rng.choice([1e-2, 1e-3, 1e-4, 1e-5])) if eb_mode == "rel" else float(rng.choice([1e-3, 0.05, 2.0]))
+    # spikes in units of 2·eb (ABS) or of the smooth part's scale (REL): around the
+    # F2I cut (|q| ~ 2^22), deep in F2I territory (2^26), and a RANGE hit in 1 seed of 8
+    unit = 2 * eb if eb_mode == "abs" else np.abs(base).max() + 1.0
+    big = [2**22 - 0.5, 2**22 + 0.5, -(2**22 + 1.5), 2**26 + 3, 3e5] if eb_mode == "abs" else [1e3, -5e2, 37.0]
+    if seed % 8 == 7:
+        big.append(2**31 if eb_mode == "abs" else np.inf)
+    k = rng.integers(0, n, max(1, n // 200))
+    x[k] = rng.choice([0.0, -0.0, 1e-40, -1e-40] + [b * unit for b in big], size=k.size)
+    xh = x.astype(dtype)
+    check_roundtrip(xh, eb, eb_mode, "outlier" if seed % 4 < 2 else "plain")
