@@ -381,3 +381,40 @@ def test_randomized_parity(seed):
     x[k] = rng.choice([0.0, -0.0, 1e-40, -1e-40] + [b * unit for b in big], size=k.size)
     xh = x.astype(dtype)
     check_roundtrip(xh, eb, eb_mode, "outlier" if seed % 4 < 2 else "plain")
+
+
+def test_c_abi_rejects_invalid_arguments():
+    """include/cszp2.h error behaviour: every entry point returns CSZP2_ERR_ARG (and
+    touches nothing) for null / misaligned pointers, unknown dtype / modes / flags,
+    non-positive or non-finite bounds and oversized n."""
+    import ctypes
+
+    L = cz._lib
+    x = torch.zeros(4096, dtype=torch.float32, device=DEV)
+    out = torch.zeros(cz.compress_bound(4096) + 64, dtype=torch.uint8, device=DEV)
+    nb = torch.zeros(1, dtype=torch.int64, device=DEV)
+    p = lambda t, off=0: ctypes.c_void_p(t.data_ptr() + off)  # noqa: E731
+    s = ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
+    E = cz.ERR_ARG
+    assert L.cszp2_compress(None, 10, 0, 1e-3, 0, 0, p(out), p(nb), s) == E          # null input
+    assert L.cszp2_compress(p(x), 10, 0, 1e-3, 0, 0, None, p(nb), s) == E            # null output
+    assert L.cszp2_compress(p(x), 10, 2, 1e-3, 0, 0, p(out), p(nb), s) == E          # dtype
+    assert L.cszp2_compress(p(x), 10, 0, 1e-3, 2, 0, p(out), p(nb), s) == E          # eb_mode
+    assert L.cszp2_compress(p(x), 10, 0, 1e-3, 0, 2, p(out), p(nb), s) == E          # enc_mode
+    for eb in (0.0, -1.0, float("nan"), float("inf")):
+        assert L.cszp2_compress(p(x), 10, 0, eb, 0, 0, p(out), p(nb), s) == E        # bound
+    assert L.cszp2_compress(p(x, 4), 10, 0, 1e-3, 0, 0, p(out), p(nb), s) == E       # misaligned in
+    assert L.cszp2_compress(p(x), 10, 0, 1e-3, 0, 0, p(out, 8), p(nb), s) == E       # misaligned out
+    assert L.cszp2_compress(p(x), (1 << 40) + 1, 0, 1e-3, 0, 0, p(out), p(nb), s) == E  # n too large
+    assert L.cszp2_compress_encode_ex(p(x), 10, 0, 1e-3, 0, 0, p(out), p(nb), 8, s) == E  # flags
+    assert L.cszp2_compress_encode_ex(p(x), 10, 0, 1e-3, 0, 0, p(out), p(nb), 6, s) == E  # vec+scalar
+    assert L.cszp2_decompress(None, p(x), 10, 0, None, s) == E
+    assert L.cszp2_decompress(p(out), p(x, 4), 10, 0, None, s) == E
+    assert L.cszp2_decompress(p(out), p(x), 10, 3, None, s) == E
+    assert L.cszp2_value_range(p(x), 10, 0, None, s) == E
+    assert L.cszp2_value_range(p(x), 10, 0, p(out, 8), s) == E
+    assert L.cszp2_compress_prepare_range(p(x), 10, 0, 1e-3, None, p(out), s) == E
+    assert L.cszp2_compress_prepare_range(p(x), 10, 0, 1e-3, p(out, 8), p(out), s) == E
+    assert L.cszp2_compress_prepare_range(p(x), 10, 0, 0.0, p(nb), p(out), s) == E
+    torch.cuda.synchronize()
+    assert int(nb.item()) == 0 and int(out.sum().item()) == 0  # nothing was written
