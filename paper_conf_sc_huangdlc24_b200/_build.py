@@ -21,6 +21,7 @@ NVCC_FLAGS = [
 
 def sources():
     return sorted(glob.glob(os.path.join(CSRC, "*.cu")) + glob.glob(os.path.join(CSRC, "*.cuh"))
+                  + glob.glob(os.path.join(CSRC, "*.cpp"))
                   + [os.path.join(ROOT, "include", "cszp2.h")])
 
 
@@ -33,7 +34,23 @@ def build(force: bool = False, verbose: bool = False) -> str:
         cmd.insert(1, "-Xptxas=-v")
     subprocess.check_call(cmd)
     os.replace(LIB + ".tmp", LIB)
+    build_cli()
     return LIB
+
+
+CLI = os.path.join(PKG, "cszp2")
+
+
+def build_cli() -> str:
+    """The `cszp2` command-line tool (csrc/cszp2_cli.cpp): host C++ over the C ABI,
+    linked against the in-tree libcszp2.so (rpath $ORIGIN) and cudart."""
+    cuda = os.path.dirname(os.path.dirname(os.path.realpath(NVCC)))
+    cmd = ["g++", "-O2", "-std=c++17", "-I", os.path.join(ROOT, "include"), "-I", os.path.join(cuda, "include"),
+           "-o", CLI + ".tmp", os.path.join(CSRC, "cszp2_cli.cpp"), "-L", PKG, "-lcszp2",
+           "-L", os.path.join(cuda, "lib64"), "-lcudart", "-Wl,-rpath,$ORIGIN"]
+    subprocess.check_call(cmd)
+    os.replace(CLI + ".tmp", CLI)
+    return CLI
 
 
 if __name__ == "__main__":
