@@ -291,6 +291,10 @@ def main():
     prep_ms, enc_ms, gather_ms, dec_ms = ph.mean(axis=0)
     comp_ms = prep_ms + enc_ms + gather_ms
     stream_bytes = int(nbytes.item())
+    # per-step spread (median and min next to the mean), this rank
+    comp_steps, dec_steps = ph[:, 0] + ph[:, 1] + ph[:, 2], ph[:, 3]
+    spread = {"comp_ms_median": round(float(np.median(comp_steps)), 4), "comp_ms_min": round(float(comp_steps.min()), 4),
+              "decomp_ms_median": round(float(np.median(dec_steps)), 4), "decomp_ms_min": round(float(dec_steps.min()), 4)}
 
     # max over ranks of every timing (device clocks), sum of stream bytes
     vec = torch.tensor([total_ms, comp_ms, dec_ms, prep_ms, enc_ms, gather_ms], dtype=torch.float64, device=dev)
@@ -368,6 +372,27 @@ def main():
         step()  # leave the main-mode stream in `out`
         torch.cuda.synchronize()
 
+    # ABS mode with eb = the REL run's eb_abs: the same quantization without the
+    # min/max pass, so the cost of REL's extra read is visible
+    abs_mode = None
+    if spec.eb_mode == "rel":
+        eb_abs = cz.read_header(out)["eb_abs"]
+        ae = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(4)]
+        for k in range(6):
+            if k >= 2:
+                ae[k - 2][0].record(stream)
+            cz.compress(x, eb_abs, "abs", args.enc, out=out, out_bytes=nbytes, stream=stream)
+            if k >= 2:
+                ae[k - 2][1].record(stream)
+        torch.cuda.synchronize()
+        av = torch.tensor([float(np.mean([e[0].elapsed_time(e[1]) for e in ae]))], dtype=torch.float64, device=dev)
+        if dist:
+            dist.all_reduce(av, op=dist.ReduceOp.MAX)
+        abs_mode = {"comp_gbs": round(gb_field / (av.item() * 1e-3), 1), "eb": "eb_abs of the REL run (per rank)",
+                    "note": "memset + compress kernel; REL adds the min/max read (phase_ms.prepare_minmax)"}
+        step()  # leave the main-mode stream in `out`
+        torch.cuda.synchronize()
+
     # cpu_baseline: the oracle as it stands, on a bounded sample, rank 0 at N=1 only
     cpu = cpu_mt = None
     if rank == 0 and world == 1:
@@ -397,6 +422,8 @@ def main():
             "eb_abs_rank0": hdr["eb_abs"],
             "phase_ms": {"prepare_minmax": round(prep_ms, 4), "compress_kernel": round(enc_ms, 4),
                          "allgather_index": round(gather_ms, 4), "decompress_kernel": round(dec_ms, 4)},
+            "step_spread_rank0": spread,
+            "abs_mode": abs_mode,
             "roofline": roof,
             "cpu_baseline": cpu,
             "cpu_baseline_all_cores": cpu_mt,
