@@ -157,6 +157,19 @@ def traffic_from_profiles(kernel_key: str):
         return None
 
 
+def workload_config(args, spec, lam, world, n_total, values_per_rank):
+    """The `config` object of both arms (the reference arm times a sample of it)."""
+    return {"workload": f"{args.config}: {spec.name} {spec.dtype} field, REL {lam:g}, "
+                        f"{args.enc}-FLE, slab-sharded over {world} rank(s)",
+            "n_values": n_total, "values_per_rank": values_per_rank, "eb_mode": spec.eb_mode,
+            "eb": lam, "enc_mode": args.enc,
+            "l2": "inputs larger than L2 (field >> 126 MB); no flush needed",
+            "rel_scope": args.rel_scope,
+            "parallelism": f"slab x{world}, NCCL all-gather of compressed sizes"
+                           + (" + all-reduce of the value range"
+                              if args.rel_scope == "global" and spec.eb_mode == "rel" else "")}
+
+
 # ----------------------------------------------------------------- reference arm (CPU oracle)
 
 def run_reference(args):
@@ -195,8 +208,10 @@ def run_reference(args):
         "ms_per_step": round((tc + td) / args.steps * 1e3, 3), "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f32" if w == 4 else "f64",
         "data": "synthetic",
-        "config": {"workload": f"{args.config} {spec.name} REL {lam:g} {args.enc} (oracle sample)",
-                   "sample_values": sample},
+        # rank 0's slab size, computed here (this arm loads nothing of the product)
+        "config": workload_config(args, spec, lam, world, spec.n,
+                                  min(spec.n, -(-(-(-spec.n // world)) // 32) * 32)),
+        "reference_sample_values": sample,
         "comp_gbs": round(gb / tc, 4), "decomp_gbs": round(gb / td, 4),
         "cr": round(x.nbytes / s.size, 3),
         "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
@@ -409,14 +424,7 @@ def main():
             "ms_per_step": round(total_ms / args.steps, 4), "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None,
             "dtype": "f32" if w == 4 else "f64", "data": "synthetic",
-            "config": {"workload": f"{args.config}: {spec.name} {spec.dtype} field, REL {lam:g}, "
-                                   f"{args.enc}-FLE, slab-sharded over {world} rank(s)",
-                       "n_values": n_total, "values_per_rank": cnt, "eb_mode": spec.eb_mode,
-                       "eb": lam, "enc_mode": args.enc,
-                       "l2": "inputs larger than L2 (field >> 126 MB); no flush needed",
-                       "rel_scope": args.rel_scope,
-                       "parallelism": f"slab x{world}, NCCL all-gather of compressed sizes"
-                                      + (" + all-reduce of the value range" if glob else "")},
+            "config": workload_config(args, spec, lam, world, n_total, cnt),
             "comp_gbs": round(comp_gbs, 1), "decomp_gbs": round(decomp_gbs, 1),
             "cr": round(n_total * w / stream_total, 3), "psnr_db": round(psnr, 3),
             "eb_abs_rank0": hdr["eb_abs"],
