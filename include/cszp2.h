@@ -21,6 +21,8 @@
  *    (status byte) and through d_status, never by the return value.
  *  - Alignment: d_in, d_out, d_cmp must be 16-byte aligned (TMA requirement);
  *    cudaMalloc'd pointers are.
+ *  - Size: the 1D entry points take n <= 2^35 values (the dense side is a tensor of
+ *    128-byte rows addressed by int32 TMA coordinates); larger n is ARG.
  */
 #ifndef CSZP2_H
 #define CSZP2_H
@@ -67,6 +69,7 @@ typedef struct {
 uint64_t cszp2_compress_bound(uint64_t n, int dtype);
 
 /* Compression (P:84-102 problem statement; Fig 4 workflow ❶-❹).
+ *  n           : number of values, 0 <= n <= 2^35 (TMA row coordinates are int32), else ARG.
  *  d_in        : n values of `dtype`, device, 16-byte aligned, read only.
  *  eb          : ABS bound, or REL lambda in (0,1); finite and > 0.
  *  d_out       : device buffer of cszp2_compress_bound(n, dtype) bytes,

@@ -105,13 +105,17 @@ unsigned persistent_grid(K kernel, int threads, int smem, uint64_t tiles, int *c
     return static_cast<unsigned>(t < static_cast<uint64_t>(*cache) ? t : *cache);
 }
 
+// Largest n of the 1D entry points: the dense side is a tensor of 128-byte rows (n/32
+// rows for f32, n/16 for f64) and TMA coordinates are int32, so rows stay below 2^31.
+constexpr uint64_t MAX_N = 1ull << 35;
+
 int check_compress_args(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
                         const void *d_out) {
     if (!wsize(dtype) || !d_out || (!d_in && n)) return CSZP2_ERR_ARG;
     if (eb_mode != CSZP2_EB_ABS && eb_mode != CSZP2_EB_REL) return CSZP2_ERR_ARG;
     if (!(eb > 0.0) || !std::isfinite(eb)) return CSZP2_ERR_ARG;
     if (!aligned16(d_out) || (n && !aligned16(d_in))) return CSZP2_ERR_ARG;
-    if (n > (1ull << 40)) return CSZP2_ERR_ARG;  // TMA row coordinates are int32
+    if (n > MAX_N) return CSZP2_ERR_ARG;
     return CSZP2_OK;
 }
 
@@ -308,7 +312,7 @@ int cszp2_compress_prepare(const void *d_in, uint64_t n, int dtype, double eb, i
 
 int cszp2_value_range(const void *d_in, uint64_t n, int dtype, double *d_work, void *stream) {
     if (!wsize(dtype) || !d_work || (!d_in && n)) return CSZP2_ERR_ARG;
-    if ((n && !aligned16(d_in)) || !aligned16(d_work) || n > (1ull << 40)) return CSZP2_ERR_ARG;
+    if ((n && !aligned16(d_in)) || !aligned16(d_work) || n > MAX_N) return CSZP2_ERR_ARG;
     // d_work[0..1]: the result; bytes 32..63: the reduction's header-shaped scratch
     if (cudaMemsetAsync(d_work, 0, 8 * sizeof(double), S(stream)) != cudaSuccess) return CSZP2_ERR_CUDA;
     return dtype == CSZP2_F32 ? launch_minmax<float>(d_in, n, 1.0, d_work, S(stream), d_work)
@@ -365,7 +369,7 @@ int cszp2_decompress(const void *d_cmp, void *d_out, uint64_t n, int dtype, int 
                      void *stream) {
     if (!wsize(dtype) || !d_cmp || (!d_out && n)) return CSZP2_ERR_ARG;
     if (!aligned16(d_cmp) || (n && !aligned16(d_out))) return CSZP2_ERR_ARG;
-    if (n > (1ull << 40)) return CSZP2_ERR_ARG;
+    if (n > MAX_N) return CSZP2_ERR_ARG;
     Geom g = geometry(n);
     return dtype == CSZP2_F32 ? launch_decompress<float>(d_cmp, d_out, g, d_status, S(stream))
                               : launch_decompress<double>(d_cmp, d_out, g, d_status, S(stream));
@@ -380,7 +384,7 @@ int cszp2_decompress_tilewise(const void *d_cmp, void *d_out, uint64_t n, int dt
                               void *d_scratch, int *d_status, void *stream) {
     if (!wsize(dtype) || !d_cmp || !d_scratch || (!d_out && n)) return CSZP2_ERR_ARG;
     if (locate != CSZP2_LOCATE_INDEX && locate != CSZP2_LOCATE_LOOKBACK) return CSZP2_ERR_ARG;
-    if (!aligned16(d_cmp) || (n && !aligned16(d_out)) || n > (1ull << 40)) return CSZP2_ERR_ARG;
+    if (!aligned16(d_cmp) || (n && !aligned16(d_out)) || n > MAX_N) return CSZP2_ERR_ARG;
     const Geom g = geometry(n);
     cudaStream_t st = S(stream);
     if (cudaMemsetAsync(d_scratch, 0, cszp2_decompress_scratch_bytes(n), st) != cudaSuccess)
@@ -408,7 +412,7 @@ int cszp2_decompress_tilewise(const void *d_cmp, void *d_out, uint64_t n, int dt
 int cszp2_decompress_range(const void *d_cmp, uint64_t n, int dtype, uint64_t first,
                            uint64_t count, void *d_out, int *d_status, void *stream) {
     if (!wsize(dtype) || !d_cmp || (!d_out && count)) return CSZP2_ERR_ARG;
-    if (!aligned16(d_cmp) || n > (1ull << 40) || first > n || count > n - first) return CSZP2_ERR_ARG;
+    if (!aligned16(d_cmp) || n > MAX_N || first > n || count > n - first) return CSZP2_ERR_ARG;
     if (count == 0) return CSZP2_OK;
     Geom g = geometry(n);
     const uint64_t t0 = (first / L) / BPT, t1 = ((first + count - 1) / L) / BPT;
