@@ -498,6 +498,17 @@ def run_e2e(args, cz, x, y, out, dev, stream, lam, spec, dist, world, n_total, w
     return res
 
 
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
 def run_cpu_baseline(args, x, lam, spec):
     import oracle
 
@@ -505,13 +516,24 @@ def run_cpu_baseline(args, x, lam, spec):
     xs = x[:m].cpu().numpy()
     ebm = oracle.REL if spec.eb_mode == "rel" else oracle.ABS
     enc = oracle.OUTLIER if args.enc == "outlier" else oracle.PLAIN
-    t0 = time.perf_counter()
-    s, rc = oracle.compress(xs, lam, ebm, enc)
-    t1 = time.perf_counter()
-    yh, rc2 = oracle.decompress(s, m, xs.dtype)
-    t2 = time.perf_counter()
+    # pinned to one core for the single-threaded run, restored afterwards
+    try:
+        aff = os.sched_getaffinity(0)
+        os.sched_setaffinity(0, {max(aff)})
+    except (AttributeError, OSError):
+        aff = None
+    try:
+        t0 = time.perf_counter()
+        s, rc = oracle.compress(xs, lam, ebm, enc)
+        t1 = time.perf_counter()
+        yh, rc2 = oracle.decompress(s, m, xs.dtype)
+        t2 = time.perf_counter()
+    finally:
+        if aff:
+            os.sched_setaffinity(0, aff)
     gb = xs.nbytes / 1e9
     return {"value": round(gb / (t2 - t0), 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+            "cpu": cpu_model(), "pinned": aff is not None,
             "comp_gbs": round(gb / (t1 - t0), 4), "decomp_gbs": round(gb / (t2 - t1), 4),
             "seconds": round(t2 - t0, 2),
             "sample": f"first {m} values ({xs.nbytes / 2**30:.2f} GiB) of the rank-0 slab, one "
@@ -544,7 +566,7 @@ def run_cpu_baseline_all_cores(args, x, lam, spec):
         t2 = time.perf_counter()
     gb = xs.nbytes / 1e9
     return {"value": round(gb / (t2 - t0), 4), "unit": "GB/s", "cores": min(cores, len(chunks)),
-            "kind": "oracle", "comp_gbs": round(gb / (t1 - t0), 4), "decomp_gbs": round(gb / (t2 - t1), 4),
+            "kind": "oracle", "cpu": cpu_model(), "comp_gbs": round(gb / (t1 - t0), 4), "decomp_gbs": round(gb / (t2 - t1), 4),
             "seconds": round(t2 - t0, 2),
             "sample": f"the cpu_baseline sample in {len(chunks)} block-aligned chunks, one oracle "
                       f"thread per core (REL range by one serial oracle pass)"}
