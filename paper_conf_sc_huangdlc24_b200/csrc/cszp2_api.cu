@@ -236,7 +236,8 @@ int launch_compress_nd(const void *d_in, const GeomND &g, double eb, int eb_mode
                        void *d_out, uint64_t *d_out_bytes, cudaStream_t st) {
     static std::once_flag once;
     static int attr_rc = CSZP2_OK;
-    constexpr int smem = ND_STAGE + 64;
+    static int grid_cache = 0;
+    constexpr int smem = ND_RING + 64;
     std::call_once(once, [] { attr_rc = set_smem(compress_nd_kernel<T, NDIM, OUTLIER>, smem); });
     if (attr_rc) return attr_rc;
     unsigned *ticket = reinterpret_cast<unsigned *>(static_cast<uint8_t *>(d_out) + stream_bound_nd(g));
@@ -246,7 +247,7 @@ int launch_compress_nd(const void *d_in, const GeomND &g, double eb, int eb_mode
     hs.eb_mode = static_cast<uint32_t>(eb_mode);
     hs.eb_user = eb;
     hs.flags = 0;
-    const unsigned grid = static_cast<unsigned>(g.T ? g.T : 1);
+    const unsigned grid = persistent_grid(compress_nd_kernel<T, NDIM, OUTLIER>, NT, smem, g.T, &grid_cache);
     compress_nd_kernel<T, NDIM, OUTLIER><<<grid, NT, smem, st>>>(
         static_cast<const T *>(d_in), g, eb, eb_mode == CSZP2_EB_REL ? 1 : 0,
         static_cast<uint8_t *>(d_out), ticket, d_out_bytes, hs);

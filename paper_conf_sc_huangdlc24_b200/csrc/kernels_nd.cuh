@@ -114,18 +114,29 @@ __device__ __forceinline__ void put_word(uint8_t *base, uint32_t pos, uint32_t w
     }
 }
 
-constexpr uint32_t ND_STAGE = BPT * 4 * LND + 64;  // max tile payload + slack
+constexpr uint32_t ND_STAGE = BPT * 4 * LND + 64;  // max tile payload + slack (decompression)
+constexpr uint32_t ND_TILE_MAX = BPT * 4 * LND;      // largest tile payload (Plain, fl = 31)
+constexpr uint32_t ND_RING = 96 * 1024;              // compression staging ring (>= ND_TILE_MAX)
 
+// Persistent compression CTAs (2 per SM), one thread per 64-value block, tiles claimed
+// in order from an atomic ticket. The decoupled lookback of a tile is DEFERRED by one
+// tile: iteration k encodes and stages tile t_k and publishes its aggregate, then
+// finishes the lookback of t_{k-1} (its window loads were issued at the end of iteration
+// k-1, so their latency hid behind t_k's gather and encode) and writes t_{k-1}'s payload
+// from the staging ring. A claimed tile therefore never waits on any lookback before
+// publishing its aggregate (no deadlock: every predecessor publishes unconditionally),
+// and no CTA idles on the inclusive-prefix round trip. When the ring cannot hold both
+// payloads, t_{k-1} is resolved and written first.
 template <typename T, int NDIM, bool OUTLIER>
-__global__ void __launch_bounds__(NT) compress_nd_kernel(const T *__restrict__ in, const GeomND g,
-                                                         const double eb_abs_arg,
-                                                         const int eb_from_header,
-                                                         uint8_t *__restrict__ out,
-                                                         unsigned *__restrict__ ticket,
-                                                         uint64_t *__restrict__ d_out_bytes,
-                                                         const HdrStatic hs) {
+__global__ void __launch_bounds__(NT, 2) compress_nd_kernel(const T *__restrict__ in, const GeomND g,
+                                                            const double eb_abs_arg,
+                                                            const int eb_from_header,
+                                                            uint8_t *__restrict__ out,
+                                                            unsigned *__restrict__ ticket,
+                                                            uint64_t *__restrict__ d_out_bytes,
+                                                            const HdrStatic hs) {
     extern __shared__ uint8_t stage_raw[];
-    uint8_t *stage = smem_align<16>(stage_raw);
+    uint8_t *ring = smem_align<16>(stage_raw);
     __shared__ uint32_t s_warp[NT / 32];
     __shared__ uint32_t s_tk;
     __shared__ uint64_t s_excl;
@@ -133,169 +144,207 @@ __global__ void __launch_bounds__(NT) compress_nd_kernel(const T *__restrict__ i
     const int tid = threadIdx.x;
     const uint64_t T_eff = g.T ? g.T : 1;
     uint64_t *index = reinterpret_cast<uint64_t *>(out + 64);
-    if (tid == 0) s_tk = atomicAdd(ticket, 1u);  // in-order tiles: forward progress
-    __syncthreads();
-    const uint64_t t = s_tk;
     const double eb_abs =
         eb_from_header ? *reinterpret_cast<const volatile double *>(out + 32) : eb_abs_arg;
     const auto K = make_consts(eb_abs, static_cast<T *>(nullptr));
 
-    const uint64_t b = t * BPT + tid;
-    const bool active = b < g.nb;
-    // ---- gather + ❶ quantize; values outside the field stay 0 and get residual 0
-    int q[LND];
-    uint64_t outside = 0;  // bit i: value i lies outside the field
-    bool bad = false;
-    const BlockOrigin bo = block_origin<NDIM>(g, active ? b : 0);
-    if (active && interior_vec<T, NDIM>(g, bo)) {
-        // interior block: each row of BX values by 16-byte loads
-        using S = BlockShape<NDIM>;
-        using VT = typename Vec16<T>::type;
-        constexpr int V = Vec16<T>::V;
-#pragma unroll
-        for (int r = 0; r < S::BY * S::BZ; r++) {
-            const int iy = r % S::BY, iz = r / S::BY;
-            const VT *row = reinterpret_cast<const VT *>(
-                in + ((bo.z0 + iz) * g.ny + bo.y0 + iy) * g.nx + bo.x0);
-#pragma unroll
-            for (int v = 0; v < S::BX / V; v++) {
-                T tmp[V];
-                *reinterpret_cast<VT *>(tmp) = __ldg(row + v);
-#pragma unroll
-                for (int k = 0; k < V; k++) q[r * S::BX + v * V + k] = quantize_nd<NDIM>(tmp[k], K.inv, bad);
+    // the deferred tile (uniform in the CTA): its number, aggregate, range flag and
+    // ring position; warp 0 also holds its lookback window
+    bool have_prev = false;
+    uint64_t prev_t = 0;
+    uint32_t prev_agg = 0, prev_pos = 0;
+    bool prev_bad = false;
+    LookbackWindow w;
+
+    // resolve the deferred tile (warp 0: lookback; tile 0 / no index: 0), write its
+    // payload from the ring, and for the last tile the pads, header and d_out_bytes
+    auto flush_prev = [&]() {
+        if (tid < 32) {
+            bool rng = prev_bad;
+            uint64_t e = 0;
+            if (g.T && prev_t > 0) e = lookback_finish(index, prev_t, prev_agg, prev_bad, w, &rng);
+            if (tid == 0) {
+                s_excl = e;
+                s_rng = rng;
             }
         }
-    } else {
-#pragma unroll
-        for (int i = 0; i < LND; i++) {
-            const uint64_t idx = active ? nd_index<NDIM>(g, bo, i) : ~uint64_t(0);
-            q[i] = 0;
-            if (idx != ~uint64_t(0))
-                q[i] = quantize_nd<NDIM>(in[idx], K.inv, bad);
-            else
-                outside |= 1ull << i;
+        __syncthreads();  // s_excl visible; the ring bytes of the deferred tile are complete
+        const uint64_t dst0 = g.D + s_excl;
+        write_payload(ring + (prev_pos % ND_RING), out, dst0, prev_agg, tid, NT);
+        if (prev_t == T_eff - 1) {  // last tile: pads, header, d_out_bytes
+            const uint64_t dst1 = dst0 + prev_agg;
+            if (tid >= 32 && tid < 48) {
+                const uint64_t o = dst1 + (tid - 32);
+                if (o < roundup16(dst1)) out[o] = 0;
+            }
+            if (tid >= 64 && tid < 80) {
+                const uint64_t o = g.O + g.nb + (tid - 64);
+                if (o < g.D) out[o] = 0;
+            }
+            if (tid == 0) {
+                const uint32_t status = s_rng ? ST_RANGE : 0u;
+                const uint64_t pb = status ? 0 : s_excl + prev_agg;
+                const uint64_t total = roundup16(g.D + pb);
+                uint64_t *h = reinterpret_cast<uint64_t *>(out);
+                h[0] = MAGIC | (static_cast<uint64_t>(hs.word1) << 32);
+                h[1] = hs.eb_mode | (status << 8) | (static_cast<uint64_t>(BPT) << 16) |
+                       (static_cast<uint64_t>(NDIM - 1) << 32);
+                h[2] = g.n;
+                h[3] = static_cast<uint64_t>(__double_as_longlong(hs.eb_user));
+                h[4] = static_cast<uint64_t>(__double_as_longlong(eb_abs));
+                h[5] = pb;
+                h[6] = total;
+                h[7] = g.nx | (g.ny << 32);
+                if (d_out_bytes) *d_out_bytes = total;
+            }
         }
-    }
-    // ---- nD Lorenzo residuals, highest index first so every prediction still sees q
-    uint32_t a[LND];
-    uint64_t sign = 0;
-    uint32_t or_rest = 0;
-#pragma unroll
-    for (int i = LND - 1; i >= 0; i--) {
-        int d = q[i] - lorenzo_pred<NDIM>(q, i);
-        if ((outside >> i) & 1ull) d = 0;
-        a[i] = static_cast<uint32_t>(d < 0 ? -d : d);
-        sign |= static_cast<uint64_t>(d < 0) << i;
-        if (i) or_rest |= a[i];
-    }
-    // ---- ❷ FLE with 8-byte fields
-    const int fl_p = 32 - __clz(or_rest | a[0]);
-    uint32_t size = fl_p ? 8u * (1u + fl_p) : 0u;
-    uint32_t obyte = static_cast<uint32_t>(fl_p);
-    int fl = fl_p, nob = 0;
-    if (OUTLIER) {
-        const int fl_o = 32 - __clz(or_rest);
-        const int ob = max(1, (32 - __clz(a[0]) + 7) >> 3);
-        const uint32_t size_o = 8u + ob + 8u * fl_o;
-        if (size_o < size) {
-            size = size_o;
-            obyte = 0x80u | (static_cast<uint32_t>(ob - 1) << 5) | static_cast<uint32_t>(fl_o);
-            fl = fl_o;
-            nob = ob;
-        }
-    }
-    if (!active) {
-        size = 0;
-        bad = false;
-    }
-    if (!K.ok) bad = true;
+        __syncthreads();  // the ring bytes and s_excl are free again
+        have_prev = false;
+    };
 
-    // ---- ❸ scan + decoupled lookback
-    const bool any_bad = __syncthreads_or(bad);
-    uint32_t agg;
-    const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg);
-    if (tid < 32) {
-        bool rng = any_bad;
-        uint64_t e = 0;
-        if (g.T) {
-            if (tid == 0) publish_aggregate(index, t, agg, any_bad);
-            __syncwarp();
-            if (t > 0) e = lookback(index, t, agg, any_bad, &rng);
-        }
-        if (tid == 0) {
-            s_excl = e;
-            s_rng = rng;
-        }
-    }
-    if (active) out[g.O + b] = static_cast<uint8_t>(obyte);
+    for (;;) {
+        if (tid == 0) s_tk = atomicAdd(ticket, 1u);  // in-order tiles: forward progress
+        __syncthreads();
+        const uint64_t t = s_tk;
+        if (t >= T_eff) break;
 
-    // ---- payload into the stage: sign (8 B), outlier (nob B), planes (8 B each:
-    //      values 0..31 then 32..63), bit planes by two in-register transposes
-    const uint32_t outl = a[0];
-    if (OUTLIER && nob) a[0] = 0;
-    uint32_t(&lo)[32] = *reinterpret_cast<uint32_t(*)[32]>(&a[0]);   // values 0..31
-    uint32_t(&hi)[32] = *reinterpret_cast<uint32_t(*)[32]>(&a[32]);  // values 32..63
-    const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, static_cast<unsigned>(size ? fl : 0)));
-    if (flw > 0) {
-        if (flw <= 4) {
-            pack_planes<2>(lo);
-            pack_planes<2>(hi);
-        } else if (flw <= 8) {
-            pack_planes<3>(lo);
-            pack_planes<3>(hi);
-        } else if (flw <= 16) {
-            pack_planes<4>(lo);
-            pack_planes<4>(hi);
+        const uint64_t b = t * BPT + tid;
+        const bool active = b < g.nb;
+        // ---- gather + ❶ quantize; values outside the field stay 0 and get residual 0
+        int q[LND];
+        uint64_t outside = 0;  // bit i: value i lies outside the field
+        bool bad = false;
+        const BlockOrigin bo = block_origin<NDIM>(g, active ? b : 0);
+        if (active && interior_vec<T, NDIM>(g, bo)) {
+            // interior block: each row of BX values by 16-byte loads
+            using S = BlockShape<NDIM>;
+            using VT = typename Vec16<T>::type;
+            constexpr int V = Vec16<T>::V;
+#pragma unroll
+            for (int r = 0; r < S::BY * S::BZ; r++) {
+                const int iy = r % S::BY, iz = r / S::BY;
+                const VT *row = reinterpret_cast<const VT *>(
+                    in + ((bo.z0 + iz) * g.ny + bo.y0 + iy) * g.nx + bo.x0);
+#pragma unroll
+                for (int v = 0; v < S::BX / V; v++) {
+                    T tmp[V];
+                    *reinterpret_cast<VT *>(tmp) = __ldg(row + v);
+#pragma unroll
+                    for (int k = 0; k < V; k++) q[r * S::BX + v * V + k] = quantize_nd<NDIM>(tmp[k], K.inv, bad);
+                }
+            }
         } else {
-            pack_planes<5>(lo);
-            pack_planes<5>(hi);
-        }
-    }
-    if (size) {
-        uint32_t p = my_excl;
-        put_word(stage, p, static_cast<uint32_t>(sign));
-        put_word(stage, p + 4, static_cast<uint32_t>(sign >> 32));
-        p += 8;
-        for (int j = 0; j < nob; j++) stage[p + j] = static_cast<uint8_t>(outl >> (8 * j));
-        p += nob;
 #pragma unroll
-        for (int k = 0; k < 32; k++) {
-            if (k < fl) {
-                put_word(stage, p + 8 * k, lo[k]);
-                put_word(stage, p + 8 * k + 4, hi[k]);
+            for (int i = 0; i < LND; i++) {
+                const uint64_t idx = active ? nd_index<NDIM>(g, bo, i) : ~uint64_t(0);
+                q[i] = 0;
+                if (idx != ~uint64_t(0))
+                    q[i] = quantize_nd<NDIM>(in[idx], K.inv, bad);
+                else
+                    outside |= 1ull << i;
             }
         }
+        // ---- nD Lorenzo residuals, highest index first so every prediction still sees q
+        uint32_t a[LND];
+        uint64_t sign = 0;
+        uint32_t or_rest = 0;
+#pragma unroll
+        for (int i = LND - 1; i >= 0; i--) {
+            int d = q[i] - lorenzo_pred<NDIM>(q, i);
+            if ((outside >> i) & 1ull) d = 0;
+            a[i] = static_cast<uint32_t>(d < 0 ? -d : d);
+            sign |= static_cast<uint64_t>(d < 0) << i;
+            if (i) or_rest |= a[i];
+        }
+        // ---- ❷ FLE with 8-byte fields
+        const int fl_p = 32 - __clz(or_rest | a[0]);
+        uint32_t size = fl_p ? 8u * (1u + fl_p) : 0u;
+        uint32_t obyte = static_cast<uint32_t>(fl_p);
+        int fl = fl_p, nob = 0;
+        if (OUTLIER) {
+            const int fl_o = 32 - __clz(or_rest);
+            const int ob = max(1, (32 - __clz(a[0]) + 7) >> 3);
+            const uint32_t size_o = 8u + ob + 8u * fl_o;
+            if (size_o < size) {
+                size = size_o;
+                obyte = 0x80u | (static_cast<uint32_t>(ob - 1) << 5) | static_cast<uint32_t>(fl_o);
+                fl = fl_o;
+                nob = ob;
+            }
+        }
+        if (!active) {
+            size = 0;
+            bad = false;
+        }
+        if (!K.ok) bad = true;
+
+        // ---- ❸ intra-tile scan; publish the aggregate at once (never behind a lookback)
+        const bool any_bad = __syncthreads_or(bad);
+        uint32_t agg;
+        const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg);
+        if (tid == 0 && g.T) publish_aggregate(index, t, agg, any_bad);
+        if (active) out[g.O + b] = static_cast<uint8_t>(obyte);
+
+        // ---- ring space behind the deferred tile's payload, else resolve that one first
+        uint32_t pos = have_prev ? ((prev_pos + prev_agg + 15u) & ~15u) : 0u;
+        if ((pos % ND_RING) + agg > ND_RING) pos = (pos / ND_RING + 1) * ND_RING;
+        if (have_prev && pos + agg > prev_pos + ND_RING) {
+            flush_prev();
+            pos = 0;
+        }
+
+        // ---- payload into the ring: sign (8 B), outlier (nob B), planes (8 B each:
+        //      values 0..31 then 32..63), bit planes by two in-register transposes
+        const uint32_t outl = a[0];
+        if (OUTLIER && nob) a[0] = 0;
+        uint32_t(&lo)[32] = *reinterpret_cast<uint32_t(*)[32]>(&a[0]);   // values 0..31
+        uint32_t(&hi)[32] = *reinterpret_cast<uint32_t(*)[32]>(&a[32]);  // values 32..63
+        const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, static_cast<unsigned>(size ? fl : 0)));
+        if (flw > 0) {
+            if (flw <= 4) {
+                pack_planes<2>(lo);
+                pack_planes<2>(hi);
+            } else if (flw <= 8) {
+                pack_planes<3>(lo);
+                pack_planes<3>(hi);
+            } else if (flw <= 16) {
+                pack_planes<4>(lo);
+                pack_planes<4>(hi);
+            } else {
+                pack_planes<5>(lo);
+                pack_planes<5>(hi);
+            }
+        }
+        if (size) {
+            uint8_t *stg = ring + (pos % ND_RING);
+            uint32_t p = my_excl;
+            put_word(stg, p, static_cast<uint32_t>(sign));
+            put_word(stg, p + 4, static_cast<uint32_t>(sign >> 32));
+            p += 8;
+            for (int j = 0; j < nob; j++) stg[p + j] = static_cast<uint8_t>(outl >> (8 * j));
+            p += nob;
+#pragma unroll
+            for (int k = 0; k < 32; k++) {
+                if (k < fl) {
+                    put_word(stg, p + 8 * k, lo[k]);
+                    put_word(stg, p + 8 * k + 4, hi[k]);
+                }
+            }
+        }
+
+        // ---- the deferred tile: its window has been in flight since last iteration
+        if (have_prev) flush_prev();  // (its first barrier also completes this tile's staging)
+        else __syncthreads();
+
+        // ---- this tile becomes the deferred one; issue its lookback window now
+        have_prev = true;
+        prev_t = t;
+        prev_agg = agg;
+        prev_pos = pos;
+        prev_bad = any_bad;
+        if (tid < 32 && g.T && t > 0) lookback_issue(index, static_cast<int64_t>(t) - 1, w);
     }
-    __syncthreads();  // stage complete; s_excl visible
-    const uint64_t dst0 = g.D + s_excl;
-    write_payload(stage, out, dst0, agg, tid, NT);
-    if (t == T_eff - 1) {  // last tile: pads, header, d_out_bytes
-        const uint64_t dst1 = dst0 + agg;
-        if (tid >= 32 && tid < 48) {
-            const uint64_t o = dst1 + (tid - 32);
-            if (o < roundup16(dst1)) out[o] = 0;
-        }
-        if (tid >= 64 && tid < 80) {
-            const uint64_t o = g.O + g.nb + (tid - 64);
-            if (o < g.D) out[o] = 0;
-        }
-        if (tid == 0) {
-            const uint32_t status = s_rng ? ST_RANGE : 0u;
-            const uint64_t pb = status ? 0 : s_excl + agg;
-            const uint64_t total = roundup16(g.D + pb);
-            uint64_t *h = reinterpret_cast<uint64_t *>(out);
-            h[0] = MAGIC | (static_cast<uint64_t>(hs.word1) << 32);
-            h[1] = hs.eb_mode | (status << 8) | (static_cast<uint64_t>(BPT) << 16) |
-                   (static_cast<uint64_t>(NDIM - 1) << 32);
-            h[2] = g.n;
-            h[3] = static_cast<uint64_t>(__double_as_longlong(hs.eb_user));
-            h[4] = static_cast<uint64_t>(__double_as_longlong(eb_abs));
-            h[5] = pb;
-            h[6] = total;
-            h[7] = g.nx | (g.ny << 32);
-            if (d_out_bytes) *d_out_bytes = total;
-        }
-    }
+    if (have_prev) flush_prev();
 }
 
 template <typename T, int NDIM>
