@@ -139,3 +139,19 @@ def test_nd_error_bound_and_ratio_vs_1d(ndim):
     err = (y.double() - x.double()).abs().max().item()
     assert err <= eb_abs * (1 + 1e-6) + 1e-7 * float(x.abs().max())
     assert total < int(n1.item())
+
+
+@pytest.mark.parametrize("kind", ["smooth", "incompressible"])
+def test_nd_persistent_multi_tile_per_cta(kind):
+    """Fields with more tiles than resident compression CTAs (1024 tiles of 4x4x4 blocks,
+    2 CTAs/SM), so every CTA defers lookbacks across several tiles; the incompressible
+    one (~60 KB per tile payload) forces the ring-full path (resolve the deferred tile
+    before staging). Whole streams and values must equal the oracle's."""
+    shape = (256, 256, 256)
+    if kind == "smooth":
+        xh = smooth_field(shape, 11, np.float32, noise=1e-2)
+        check_nd(xh, 1e-4, "rel", "outlier")
+    else:
+        rng = np.random.default_rng(12)
+        xh = (rng.standard_normal(shape) * 100.0).astype(np.float32)
+        check_nd(xh, 1e-5, "abs", "plain")
