@@ -899,12 +899,12 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
         if (LOAD == LOAD_TMA && b0 < g.nfull) {
             if (Traits<T>::ROWS == 1) {
                 mbar_expect_tx(&s_full, BPT * 128);
-                tma_load_2d(inbuf, &tmap, 0, static_cast<int>(b0), &s_full);
+                tma_load_2d_ef(inbuf, &tmap, 0, static_cast<int>(b0), &s_full);
             } else {
                 const bool second = (b0 + BPT / 2) < g.nfull;
                 mbar_expect_tx(&s_full, second ? 2 * BPT * 128 : BPT * 128);
-                tma_load_2d(inbuf, &tmap, 0, static_cast<int>(2 * b0), &s_full);
-                if (second) tma_load_2d(inbuf + BPT * 128, &tmap, 0, static_cast<int>(2 * b0 + BPT), &s_full);
+                tma_load_2d_ef(inbuf, &tmap, 0, static_cast<int>(2 * b0), &s_full);
+                if (second) tma_load_2d_ef(inbuf + BPT * 128, &tmap, 0, static_cast<int>(2 * b0 + BPT), &s_full);
             }
         } else {
             mbar_expect_tx(&s_full, 0);
@@ -1471,9 +1471,9 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? 3 : 2) decompress_kernel(
             if (Traits<T>::ROWS == 1) {
                 tma_store_2d(&tmap, 0, static_cast<int>(b0), ostage);
             } else {
-                tma_store_2d(&tmap, 0, static_cast<int>(2 * b0), ostage);
+                tma_store_2d_ef(&tmap, 0, static_cast<int>(2 * b0), ostage);
                 if (b0 + BPT / 2 < g.nfull)
-                    tma_store_2d(&tmap, 0, static_cast<int>(2 * b0 + BPT), ostage + BPT * 128);
+                    tma_store_2d_ef(&tmap, 0, static_cast<int>(2 * b0 + BPT), ostage + BPT * 128);
             }
             bulk_commit();
         }
