@@ -2,7 +2,8 @@
 library is loaded with its own ctypes handle, and the timed launches alternate
 library by library inside each repetition, so clock/power drift over the run hits
 all builds alike. Prints the median compress-kernel and decompress-kernel time per
-build (CUDA events around each launch) and the ratio to the first build.
+build (CUDA events around each launch; `prep` = cszp2_compress_prepare, i.e.
+the REL min/max pass for REL configs) and the ratio to the first build.
 
 usage: python scripts/ab_interleave.py cfg5[,cfg3b...] lib_a.so lib_b.so ... [--reps N]
 """
@@ -52,8 +53,11 @@ def main():
         for enc, encname in ((1, "outlier"), (0, "plain")):
             te = [[] for _ in Ls]
             td = [[] for _ in Ls]
+            tp = [[] for _ in Ls]
             for r in range(reps + 2):
                 for k, L in enumerate(Ls):
+                    ep = torch.cuda.Event(enable_timing=True)
+                    ep.record(st)
                     L.cszp2_compress_prepare(vp(x.data_ptr()), n, dt, lam, ebm, vp(out.data_ptr()), sp)
                     e0, e1, e2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
                     e0.record(st)
@@ -66,11 +70,14 @@ def main():
                     if r >= 2:
                         te[k].append(e0.elapsed_time(e1))
                         td[k].append(e1.elapsed_time(e2))
+                        tp[k].append(ep.elapsed_time(e0))
             me = [float(np.median(v)) for v in te]
             md = [float(np.median(v)) for v in td]
+            mp = [float(np.median(v)) for v in tp]
             for k, p in enumerate(libs):
                 print(f"{cfg:6s} {encname:8s} {os.path.basename(p):14s} enc {me[k]:8.4f} ms ({me[0] / me[k]:6.4f}x)"
-                      f"  dec {md[k]:8.4f} ms ({md[0] / md[k]:6.4f}x)", flush=True)
+                      f"  dec {md[k]:8.4f} ms ({md[0] / md[k]:6.4f}x)"
+                      f"  prep {mp[k]:8.4f} ms ({mp[0] / mp[k]:6.4f}x)", flush=True)
         del x, out, y
         torch.cuda.empty_cache()
 
