@@ -96,39 +96,6 @@ struct Vec16<double> {
     static constexpr int V = 2;
 };
 
-#ifndef CSZP2_ND_L2PF
-#define CSZP2_ND_L2PF 0
-#endif
-// 16-byte read-only load with an L2 prefetch-size hint (CSZP2_ND_L2PF = 128 / 256)
-__device__ __forceinline__ float4 ld_nd_row(const float4 *p) {
-#if CSZP2_ND_L2PF == 256
-    float4 v;
-    asm volatile("ld.global.nc.L2::256B.v4.f32 {%0, %1, %2, %3}, [%4];"
-                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
-    return v;
-#elif CSZP2_ND_L2PF == 128
-    float4 v;
-    asm volatile("ld.global.nc.L2::128B.v4.f32 {%0, %1, %2, %3}, [%4];"
-                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
-    return v;
-#else
-    return __ldg(p);
-#endif
-}
-__device__ __forceinline__ double2 ld_nd_row(const double2 *p) {
-#if CSZP2_ND_L2PF == 256
-    double2 v;
-    asm volatile("ld.global.nc.L2::256B.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
-    return v;
-#elif CSZP2_ND_L2PF == 128
-    double2 v;
-    asm volatile("ld.global.nc.L2::128B.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
-    return v;
-#else
-    return __ldg(p);
-#endif
-}
-
 // true if block b lies entirely inside the field and its rows are 16-byte aligned
 // (x extent a multiple of the vector width; the base is 16-byte aligned by the ABI)
 template <typename T, int NDIM>
@@ -261,7 +228,7 @@ __global__ void __launch_bounds__(NT, 2) compress_nd_kernel(const T *__restrict_
 #pragma unroll
                 for (int v = 0; v < S::BX / V; v++) {
                     T tmp[V];
-                                        *reinterpret_cast<VT *>(tmp) = ld_nd_row(row + v);
+                                        *reinterpret_cast<VT *>(tmp) = __ldg(row + v);
 #pragma unroll
                     for (int k = 0; k < V; k++) q[r * S::BX + v * V + k] = quantize_nd<NDIM>(tmp[k], K.inv, bad);
                 }
