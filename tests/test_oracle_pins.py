@@ -89,6 +89,54 @@ def test_error_bound_closed_form(orc, dtype, eb):
     assert err.max() > 0.9 * eb
 
 
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+@pytest.mark.parametrize("eb", [0.5, 1e-3, 3.7e-5])
+def test_error_bound_where_float_q_rounds(orc, dtype, eb):
+    """R-10 bound for |x / 2eb| from 2^24 up to the R-3 limit (2^30 - 64 for
+    f32), where (T)q is no longer exact in f32: x' = fl(fl(q)·s) (FORMAT.md §6.6)
+    must still land within eb of x plus the rounding of x' to T."""
+    rng = np.random.default_rng(11)
+    lo, hi = 2.0 ** 24, 2.0 ** 30 - 64
+    mag = np.exp(rng.uniform(np.log(lo), np.log(hi), 60000))
+    t = mag * rng.choice([-1.0, 1.0], mag.size)
+    x = (t * 2 * eb).astype(dtype)
+    x = x[np.abs(x.astype(np.float64) * (1.0 / (2 * eb))) < hi - 64]  # keep t strictly in range
+    s, rc = orc.compress(x, eb, orc.ABS, orc.PLAIN)
+    assert rc == orc.OK
+    y, rc = orc.decompress(s, x.size, dtype)
+    assert rc == orc.OK
+    err = np.abs(x.astype(np.float64) - y.astype(np.float64))
+    m = np.maximum(np.abs(x), np.abs(y)).astype(np.float64)
+    if dtype == np.float32:
+        bound = eb * (1 + 2.0 ** -20) + 2.0 ** -21 * m
+    else:
+        bound = eb * (1 + 2.0 ** -40) + 2.0 ** -50 * m
+    assert np.all(err <= bound)
+    # the values really are that large: |q| spans [2^24, 2^30) (numpy's own rint)
+    qa = np.abs(np.rint(x.astype(np.float64) / (2 * eb)))
+    assert qa.min() >= 2.0 ** 24 - 1 and qa.max() >= 2.0 ** 29
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_large_integers_round_trip_exactly_at_half(orc, dtype):
+    """eb = 0.5 (s = inv = 1): every f32 of magnitude >= 2^24 is an integer, so q = x and
+    x' = (T)q·1 must give x back exactly, up to the R-3 limit 2^30 - 64 (f32) /
+    2^30 - 1 (f64). A dequantizer that drops or wraps high bits of q, or converts
+    through a narrower type, fails here (FORMAT.md §6.6)."""
+    rng = np.random.default_rng(12)
+    top = 2 ** 30 - 64 if dtype == np.float32 else 2 ** 30 - 1
+    v = rng.integers(2 ** 24, top + 1, 40000).astype(np.float64)
+    v = np.concatenate([v, [2.0 ** 24, 2.0 ** 24 + 2, 2.0 ** 29 + 2.0 ** 6, top]])
+    x = (v * rng.choice([-1.0, 1.0], v.size)).astype(dtype)
+    assert np.all(np.abs(x.astype(np.float64)) <= top)
+    s, rc = orc.compress(x, 0.5, orc.ABS, orc.OUTLIER)
+    assert rc == orc.OK
+    y, rc = orc.decompress(s, x.size, dtype)
+    assert rc == orc.OK
+    iv = np.uint32 if dtype == np.float32 else np.uint64
+    np.testing.assert_array_equal(y.view(iv), x.view(iv))
+
+
 def test_range_status(orc):
     """|t| beyond 2^30-1 cannot be stored in the fl <= 31 code: RANGE."""
     x = np.array([0.0, 1.0, 3e9], dtype=np.float32)
