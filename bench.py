@@ -47,11 +47,17 @@ def parse():
     ap.add_argument("--enc", default="outlier", choices=["plain", "outlier"])
     ap.add_argument("--eb", type=float, default=None)
     ap.add_argument("--e2e-steps", type=int, default=2)
-    ap.add_argument("--e2e-max-gib", type=float, default=40.0,
-                    help="cap on the per-rank slab used for the host-buffer e2e leg")
+    ap.add_argument("--e2e-max-gib", type=float, default=8.0,
+                    help="cap on the per-rank slab used for the host-buffer e2e leg (pinned host "
+                         "memory per rank is ~3x this)")
     ap.add_argument("--cpu-sample-log2", type=int, default=28,
                     help="values in the oracle cpu_baseline sample (2^k)")
     ap.add_argument("--no-plain", action="store_true", help="skip the secondary Plain-mode pass")
+    ap.add_argument("--no-configs", action="store_true",
+                    help="skip the per-config sweep (BASELINE configs 1-4, both modes, both directions)")
+    ap.add_argument("--config-steps", type=int, default=20, help="timed steps per sweep entry")
+    ap.add_argument("--launcher-selftest", action="store_true",
+                    help="(tests) start the ranks like a real run, join a gloo group, report the world and exit")
     ap.add_argument("--rel-scope", default="rank", choices=["rank", "global"],
                     help="REL range per rank's slab (default; no extra collective) or of the whole "
                          "field (one 16-byte NCCL all-reduce of (min, -max); SURVEY 8(e))")
@@ -125,10 +131,14 @@ class ClockSampler:
         t_out = getattr(self, "t_out", float("inf")) + 0.06
         return [l for t, l in self.raw if self.t_in <= t <= t_out]
 
-    def summary(self):
+    def window(self, t0, t1):
+        """summary() of the samples taken in [t0, t1] (time.monotonic())."""
+        return self.summary([l for t, l in self.raw if t0 <= t <= t1 + 0.06])
+
+    def summary(self, lines=None):
         sm, mx, reasons = [], None, set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for l in self.lines:
+        for l in (self.lines if lines is None else lines):
             f = [x.strip() for x in l.split(",")]
             if len(f) < 9:
                 continue
@@ -146,13 +156,15 @@ class ClockSampler:
                 "samples": len(sm)}
 
 
-def traffic_from_profiles(kernel_key: str):
-    """dram read+write bytes per launch from the committed ncu --set full summary."""
-    p = os.path.join(ROOT, "profiles", "ncu_full_summary.json")
+def traffic_from_profiles(kernel_key: str, cfg: str = "cfg5", enc: str = "outlier"):
+    """dram read+write bytes per launch of `kernel_key` on (cfg, enc), from the
+    committed ncu --set full captures (profiles/ncu_traffic.json, written by
+    scripts/ncu_traffic.py); None when no capture of that workload is committed."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     try:
         with open(p) as f:
             d = json.load(f)
-        return d.get(kernel_key, {}).get("dram_bytes_per_launch")
+        return d.get(f"{cfg}/{enc}/{kernel_key}", {}).get("dram_bytes")
     except Exception:
         return None
 
@@ -176,6 +188,8 @@ def run_reference(args):
     rank, world, _ = dist_env()
     if rank != 0:
         return 0
+    if "WORLD_SIZE" not in os.environ:
+        world = args.gpus  # the same workload description as our arm at --gpus N
     import oracle
 
     spec = CONFIGS[args.config]
@@ -224,10 +238,52 @@ def run_reference(args):
 
 # ----------------------------------------------------------------- our arm
 
+def relaunch_under_torchrun(args) -> int:
+    """`python bench.py --gpus N` without a torchrun environment: start the N ranks
+    ourselves (one process per GPU, NCCL over 127.0.0.1) with the same arguments and
+    return their exit code; rank 0 prints the JSON line."""
+    import socket
+
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__), *sys.argv[1:]]
+    env = dict(os.environ, BENCH_SELF_LAUNCHED="1")
+    return subprocess.call(cmd, env=env)
+
+
+def launcher_selftest(args) -> int:
+    """The multi-rank plumbing of a real run without GPUs (tests/test_bench_launch.py):
+    every rank joins a gloo group over the torchrun environment and all-gathers its
+    rank; rank 0 prints what the group saw."""
+    import torch.distributed as dist
+
+    rank, world, local = dist_env()
+    dist.init_process_group("gloo")
+    got = [None] * world
+    dist.all_gather_object(got, {"rank": rank, "local_rank": local, "pid": os.getpid()})
+    t = torch.tensor([float(rank + 1)])
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    if rank == 0:
+        print(json.dumps({"n_gpus": world, "gpus_arg": args.gpus, "ranks": got, "max_over_ranks": t.item(),
+                          "self_launched": os.environ.get("BENCH_SELF_LAUNCHED") == "1"}), flush=True)
+    dist.destroy_process_group()
+    return 0
+
+
 def main():
     args = parse()
+    if args.gpus < 1:
+        raise SystemExit("--gpus must be >= 1")
+    if args.launcher_selftest:
+        if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+            return relaunch_under_torchrun(args)
+        return launcher_selftest(args)
     if args.impl == "reference":
-        return run_reference(args)
+        return run_reference(args)  # rank 0 only; needs no process group
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return relaunch_under_torchrun(args)
 
     import paper_conf_sc_huangdlc24_b200 as cz
     from paper_conf_sc_huangdlc24_b200.multi import reduce_range, slab
@@ -272,7 +328,7 @@ def main():
             cz.compress_prepare(x, lam, spec.eb_mode, out, stream=stream)
         if evs:
             evs[1].record(stream)
-        cz.compress_encode(x, lam, spec.eb_mode, enc, out, nbytes, stream=stream)
+        cz.compress_encode(x, lam, spec.eb_mode, enc, out, nbytes, stream=stream, prepared=True)
         if evs:
             evs[2].record(stream)
         if world > 1:
@@ -360,7 +416,7 @@ def main():
     dom = max(("compress_kernel", "decompress_kernel"), key=lambda k: kern[k]["ms"])
     roof = {"bound": "hbm", "kernel": dom, "achieved": round(kern[dom]["gbs"], 1), "peak": peak,
             "unit": "GB/s", "frac": round(kern[dom]["frac"], 4),
-            "traffic": traffic_from_profiles(dom), "peak_source": peak_src,
+            "traffic": traffic_from_profiles(dom, args.config, args.enc), "peak_source": peak_src,
             "algorithmic_bytes_per_launch": kern[dom]["bytes"],
             "kernels": {k: {"ms": round(v["ms"], 4), "gbs": round(v["gbs"], 1), "frac": round(v["frac"], 4)}
                         for k, v in kern.items()}}
@@ -408,6 +464,12 @@ def main():
         step()  # leave the main-mode stream in `out`
         torch.cuda.synchronize()
 
+    # every other BASELINE config, N=1 only (configs 1-4 are single-GPU configs)
+    sweep = None
+    if world == 1 and not args.no_configs:
+        with ClockSampler(local) as sclk:
+            sweep = run_config_sweep(args, cz, dev, stream, peak, sclk)
+
     # cpu_baseline: the oracle as it stands, on a bounded sample, rank 0 at N=1 only
     cpu = cpu_mt = None
     if rank == 0 and world == 1:
@@ -439,12 +501,109 @@ def main():
             "clocks": clocks,
             "gpu_launches": args.steps * (3 + (1 if world > 1 else 0)),
             "plain_mode": plain,
+            "configs": sweep,
         }
         print(json.dumps(line), flush=True)
     if dist:
         dist.barrier()
         dist.destroy_process_group()
     return 0
+
+
+SWEEP = ("cfg1", "cfg2", "cfg3a", "cfg3b", "cfg4a", "cfg4b")
+
+
+def field_quality(x, y, eb_abs, chunk=1 << 27):
+    """PSNR (R-16), max|x - x'| / eb_abs, values outside BASELINE's strict slack
+    eb(1+2^-20) (f32) / eb(1+2^-40) (f64), and the R-10 bound on every value."""
+    f32 = x.dtype == torch.float32
+    slack, rnd = (1 + 2.0 ** -20, 2.0 ** -21) if f32 else (1 + 2.0 ** -40, 2.0 ** -50)
+    mse = 0.0
+    mx_err = 0.0
+    strict = 0
+    ok = True
+    mn, mxv = math.inf, -math.inf
+    for c in range(0, x.numel(), chunk):
+        a, b = x[c:c + chunk].double(), y[c:c + chunk].double()
+        e = (a - b).abs()
+        mse += float((e * e).sum())
+        mx_err = max(mx_err, float(e.max()))
+        strict += int((e > eb_abs * slack).sum())
+        ok &= bool((e <= eb_abs * slack + rnd * torch.maximum(a.abs(), b.abs())).all())
+        mn, mxv = min(mn, float(a.min())), max(mxv, float(a.max()))
+    mse /= x.numel()
+    psnr = 20 * math.log10(mxv - mn) - 10 * math.log10(mse) if mse > 0 and mxv > mn else float("inf")
+    return {"psnr_db": round(psnr, 3), "max_err_over_eb": round(mx_err / eb_abs, 6),
+            "strict_slack_violations": strict, "bound_ok": ok}
+
+
+def run_config_sweep(args, cz, dev, stream, peak, clk):
+    """Every other BASELINE config on one GPU (BASELINE.md "Output"):
+    config x REL bound x encoding mode, both directions, device-timed with CUDA events
+    on the launching stream, L2 flushed (a 256 MiB write) before every timed
+    direction, since configs 1-3a fit in the 126 MB L2."""
+    rows = []
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    for cfg in SWEEP:
+        spec = CONFIGS[cfg]
+        x = make_field(cfg, dev)
+        n, w = x.numel(), x.element_size()
+        out = torch.empty(cz.compress_bound(n, x.dtype), dtype=torch.uint8, device=dev)
+        nbytes = torch.zeros(1, dtype=torch.int64, device=dev)
+        y = torch.empty_like(x)
+        for eb in spec.ebs:
+            for enc in ("plain", "outlier"):
+                K = args.config_steps
+                ev = [[torch.cuda.Event(enable_timing=True) for _ in range(5)] for _ in range(K)]
+                for k in range(3 + K):  # 3 untimed warm-up steps
+                    e = ev[k - 3] if k >= 3 else None
+                    flush.zero_()
+                    if e: e[0].record(stream)
+                    cz.compress_prepare(x, eb, spec.eb_mode, out, stream=stream)
+                    if e: e[1].record(stream)
+                    cz.compress_encode(x, eb, spec.eb_mode, enc, out, nbytes, stream=stream, prepared=True)
+                    if e: e[2].record(stream)
+                    flush.zero_()
+                    if e: e[3].record(stream)
+                    cz.decompress(out, n, x.dtype, out=y, stream=stream)
+                    if e: e[4].record(stream)
+                    if k == 2:
+                        torch.cuda.synchronize()
+                        t0 = time.monotonic()
+                torch.cuda.synchronize()
+                t1 = time.monotonic()
+                ph = np.array([[e[0].elapsed_time(e[1]), e[1].elapsed_time(e[2]), e[3].elapsed_time(e[4])]
+                               for e in ev])
+                prep, enc_ms, dec_ms = ph.mean(axis=0)
+                total = int(nbytes.item())
+                eb_abs = cz.read_header(out, stream)["eb_abs"]
+                gb = n * w / 1e9
+                kb = n * w + total  # algorithmic bytes of either kernel: field + stream
+                q = field_quality(x, y, eb_abs)
+                rows.append({
+                    "config": cfg, "field": spec.name, "n": n, "dtype": "f32" if w == 4 else "f64",
+                    "eb_mode": spec.eb_mode, "eb": eb, "eb_abs": eb_abs, "enc_mode": enc,
+                    "cr": round(n * w / total, 3), **q,
+                    "comp_gbs": round(gb / ((prep + enc_ms) * 1e-3), 1),
+                    "decomp_gbs": round(gb / (dec_ms * 1e-3), 1),
+                    "prepare_ms": round(prep, 4), "compress_kernel_ms": round(enc_ms, 4),
+                    "decompress_kernel_ms": round(dec_ms, 4),
+                    "roofline": {
+                        "bound": "hbm", "peak": peak, "unit": "GB/s",
+                        "compress_kernel": {"achieved": round(kb / (enc_ms * 1e-3) / 1e9, 1),
+                                            "frac": round(kb / (enc_ms * 1e-3) / 1e9 / peak, 4),
+                                            "algorithmic_bytes": kb,
+                                            "traffic": traffic_from_profiles("compress_kernel", cfg, enc)},
+                        "decompress_kernel": {"achieved": round(kb / (dec_ms * 1e-3) / 1e9, 1),
+                                              "frac": round(kb / (dec_ms * 1e-3) / 1e9 / peak, 4),
+                                              "algorithmic_bytes": kb,
+                                              "traffic": traffic_from_profiles("decompress_kernel", cfg, enc)},
+                    },
+                    "steps": K, "clocks": clk.window(t0, t1),
+                })
+        del x, out, y
+        torch.cuda.empty_cache()
+    return rows
 
 
 def run_e2e(args, cz, x, y, out, dev, stream, lam, spec, dist, world, n_total, w):

@@ -11,9 +11,10 @@
  *  - Plain pointers and sizes only; `stream` is a cudaStream_t passed as void*
  *    (NULL = legacy default stream). Pointers named d_* are DEVICE pointers,
  *    h_* are HOST pointers.
- *  - The caller owns every buffer; the library allocates nothing and keeps no
- *    state between calls. Calls on different streams with disjoint buffers may
- *    run concurrently.
+ *  - The caller owns every buffer; the library allocates nothing. Its only state
+ *    is a per-(kernel, device) cache of launch attributes (dynamic shared-memory
+ *    opt-in, resident-CTA count), so one process may drive several GPUs. Calls on
+ *    different streams with disjoint buffers may run concurrently.
  *  - Work is enqueued on `stream` without host synchronisation, except where
  *    a function says it synchronises.
  *  - Return value: CSZP2_OK, or a synchronous error (bad argument, CUDA launch
@@ -77,17 +78,23 @@ uint64_t cszp2_compress_bound(uint64_t n, int dtype);
  *  d_out_bytes : nullable DEVICE uint64; receives the stream's total bytes
  *                (also in the header), so a multi-GPU caller can all-gather
  *                it without a host sync.
- * Enqueues: a memset of the header+index region, the REL min/max kernel (REL
- * only), and the single fused compression kernel. */
+ * Enqueues: a zeroing kernel (header, tile index, ticket), the REL min/max kernel
+ * (REL only), and the single fused compression kernel. */
 int cszp2_compress(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
                    int enc_mode, void *d_out, uint64_t *d_out_bytes, void *stream);
 
 /* The two phases of cszp2_compress, exposed so callers (bench.py) can time
  * the dominant kernel alone. cszp2_compress == prepare then encode, with the
- * same arguments. prepare: zero the header+index region of d_out and, for
- * REL, run the device min/max reduction that writes eb_abs into the header.
- * encode: the fused kernel (❶ quantize, in-block difference, ❷ FLE, ❸
- * decoupled-lookback scan, ❹ concatenation). */
+ * same arguments.
+ * prepare: zero the header, tile index and ticket of d_out and, for REL, run the
+ *   device min/max reduction that writes eb_abs into the header.
+ * encode: zero the tile index (the lookback descriptors) and the ticket, then the
+ *   fused kernel (❶ quantize, in-block difference, ❷ FLE, ❸ decoupled-lookback
+ *   scan, ❹ concatenation). encode may be repeated on the same d_out (each call
+ *   writes the whole stream again); with eb_mode REL it quantizes with the eb_abs
+ *   the header holds, i.e. the one a preceding prepare (or prepare_range) on this
+ *   d_out wrote, or a previous encode left there (the same value). REL encode
+ *   on a d_out that never saw a prepare reads an undefined bound. */
 int cszp2_compress_prepare(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
                            void *d_out, void *stream);
 int cszp2_compress_encode(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
@@ -119,10 +126,16 @@ int cszp2_compress_prepare_range(const void *d_in, uint64_t n, int dtype, double
  *    of the TMA tensor tiles.
  *  CSZP2_FLAG_LOAD_SCALAR: each thread loads its block value by value (the
  *    non-vectorised baseline of the §VI-E memory ablation).
- *  LOAD_VEC and LOAD_SCALAR are exclusive (ARG otherwise). */
+ *  LOAD_VEC and LOAD_SCALAR are exclusive (ARG otherwise).
+ *  CSZP2_FLAG_PREPARED (not an ablation): the caller guarantees that a
+ *    cszp2_compress_prepare(_range) on this d_out precedes this call on the stream
+ *    with no encode in between, so the tile index and ticket are still zero and
+ *    encode skips re-zeroing them (one launch less; cszp2_compress uses it). With
+ *    the flag and no such prepare, the stream is undefined. */
 #define CSZP2_FLAG_CHAINED_SCAN 1u
 #define CSZP2_FLAG_LOAD_VEC 2u
 #define CSZP2_FLAG_LOAD_SCALAR 4u
+#define CSZP2_FLAG_PREPARED 8u
 int cszp2_compress_encode_ex(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
                              int enc_mode, void *d_out, uint64_t *d_out_bytes, unsigned flags,
                              void *stream);
@@ -201,7 +214,8 @@ int cszp2_container_index(const uint64_t *d_sizes, int nparts, uint64_t *d_offse
  * id and nx, ny in its header (a 1D decoder refuses it, and vice versa).
  *  field      : nx * ny (* nz) values of `dtype`, row-major with x fastest,
  *               device, 16-byte aligned. ndim = 2 requires nz = 1.
- *  extents    : nx, ny, nz < 2^32 and nx*ny*nz <= 2^40, else ARG.
+ *  extents    : nx, ny, nz < 2^32 and nx*ny*nz <= 2^35 (the 1D limit), else ARG,
+ *               for compression and decompression alike.
  * cszp2_compress_bound_nd: bytes d_out must hold (0 on bad arguments), including
  *   16 bytes of scratch past the stream, as cszp2_compress_bound.
  * cszp2_compress_nd: like cszp2_compress (same eb / eb_mode / enc_mode meaning,

@@ -41,10 +41,11 @@ class CudaCodec:
 
         return compress(x, self.eb, self.eb_mode, self.enc_mode, stream=stream)
 
-    def decompress(self, cmp: torch.Tensor, n: int, out: torch.Tensor, stream=None):
+    def decompress(self, cmp: torch.Tensor, n: int, out: torch.Tensor, status: torch.Tensor, stream=None):
+        """Decode into `out`; `status` (zeroed device int32) receives FORMAT/RANGE bits."""
         from . import decompress
 
-        decompress(cmp, n, out.dtype, out=out, stream=stream)
+        decompress(cmp, n, out.dtype, out=out, status=status, stream=stream)
 
 
 def _all_gather_bytes(recv: torch.Tensor, send: torch.Tensor, group=None):
@@ -76,8 +77,16 @@ def compressed_all_gather(x: torch.Tensor, eb: float, eb_mode: str = "rel", enc_
         raise RuntimeError("compressed stream larger than its buffer")
     recv = torch.empty(world * slot, dtype=torch.uint8, device=x.device)
     _all_gather_bytes(recv, buf[:slot], group)      # 3. the compressed payloads
+    status = torch.zeros(world, dtype=torch.int32, device=x.device)
     for r in range(world):                          # 4. P decompression kernels
-        codec.decompress(recv[r * slot:(r + 1) * slot], n, out[r * n:(r + 1) * n])
+        codec.decompress(recv[r * slot:(r + 1) * slot], n, out[r * n:(r + 1) * n], status[r:r + 1])
+    bad = [(r, int(v)) for r, v in enumerate(status.tolist()) if v]  # host sync after the decodes
+    if bad:
+        # a rank's shard was out of range (NaN/Inf, |x/2eb| > 2^30-1: header status RANGE)
+        # or its stream did not decode: its slice of `out` is not valid data
+        from . import CszpError
+
+        raise CszpError(f"compressed_all_gather: rank {bad[0][0]}'s stream", bad[0][1])
     if stats is not None:
         stats.update(sizes=sizes.tolist(), slot=slot, wire_bytes=world * slot, raw_bytes=world * n * w)
     return out

@@ -7,7 +7,9 @@
 
 #include <cstdio>
 #include <cstring>
+#include <map>
 #include <mutex>
+#include <utility>
 
 #include "cszp2.h"
 #include "kernels.cuh"
@@ -67,12 +69,33 @@ int make_tmap(CUtensorMap *m, const void *base, int dtype, uint64_t nfull) {
     return r == CUDA_SUCCESS ? CSZP2_OK : CSZP2_ERR_CUDA;
 }
 
+// Per-device launch state. cudaFuncSetAttribute and the occupancy query act on the
+// current device's context, so both are cached per (kernel, device): a process that
+// drives several GPUs gets the attribute set on each of them.
+int current_device() {
+    int d = 0;
+    cudaGetDevice(&d);
+    return d;
+}
+struct LaunchCache {
+    int attr_rc = -1;  // -1: not yet set on this device
+    int grid = 0;      // resident CTAs (occupancy x SMs) on this device
+};
+LaunchCache &launch_cache(const void *kernel, int dev) {
+    static std::mutex mu;
+    static std::map<std::pair<const void *, int>, LaunchCache> m;
+    std::lock_guard<std::mutex> lk(mu);
+    return m[{kernel, dev}];  // std::map references stay valid across inserts
+}
+// Opt the kernel into `bytes` of dynamic shared memory on the current device (once).
 template <typename K>
 int set_smem(K kernel, int bytes) {
-    return cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) ==
-                   cudaSuccess
-               ? CSZP2_OK
-               : CSZP2_ERR_CUDA;
+    LaunchCache &c = launch_cache(reinterpret_cast<const void *>(kernel), current_device());
+    if (c.attr_rc < 0)
+        c.attr_rc = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) == cudaSuccess
+                        ? CSZP2_OK
+                        : CSZP2_ERR_CUDA;
+    return c.attr_rc;
 }
 
 int launch_status() { return cudaGetLastError() == cudaSuccess ? CSZP2_OK : CSZP2_ERR_CUDA; }
@@ -80,29 +103,40 @@ int launch_status() { return cudaGetLastError() == cudaSuccess ? CSZP2_OK : CSZP
 // stream bound without the 16-byte scratch tail (FORMAT.md §2)
 uint64_t stream_bound(const Geom &g) { return roundup16(g.D + static_cast<uint64_t>(4 * L) * g.nb); }
 
+int sm_count();
+// zero bytes [from, to) of d_out (8-byte multiples) and the tile ticket at stream_bound
+int zero_scratch(void *d_out, uint64_t from, uint64_t to, const Geom &g, cudaStream_t st) {
+    const uint64_t words = (to - from) / 8;
+    const uint64_t want = (words + 255) / 256;
+    const uint64_t cap = 4ull * sm_count();
+    const unsigned zg = static_cast<unsigned>(want < 1 ? 1 : (want > cap ? cap : want));
+    uint8_t *o = static_cast<uint8_t *>(d_out);
+    zero_scratch_kernel<<<zg, 256, 0, st>>>(reinterpret_cast<uint64_t *>(o + from), words,
+                                            reinterpret_cast<uint4 *>(o + stream_bound(g)));
+    return cudaGetLastError() == cudaSuccess ? CSZP2_OK : CSZP2_ERR_CUDA;
+}
+
 int sm_count() {
-    static int sms = 0;
-    if (!sms) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        if (sms <= 0) sms = 148;
-    }
+    int sms = 0;
+    if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, current_device()) != cudaSuccess || sms <= 0)
+        sms = 148;
     return sms;
 }
 
-// persistent grid: every CTA resident (occupancy x SMs), never more than tiles
+// persistent grid: every CTA resident (occupancy x SMs of the current device), never
+// more than tiles
 template <typename K>
-unsigned persistent_grid(K kernel, int threads, int smem, uint64_t tiles, int *cache) {
-    if (*cache <= 0) {
+unsigned persistent_grid(K kernel, int threads, int smem, uint64_t tiles) {
+    LaunchCache &c = launch_cache(reinterpret_cast<const void *>(kernel), current_device());
+    if (c.grid <= 0) {
         int per_sm = 0;
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, smem) != cudaSuccess ||
             per_sm < 1)
             per_sm = 1;
-        *cache = per_sm * sm_count();
+        c.grid = per_sm * sm_count();
     }
     const uint64_t t = tiles ? tiles : 1;
-    return static_cast<unsigned>(t < static_cast<uint64_t>(*cache) ? t : *cache);
+    return static_cast<unsigned>(t < static_cast<uint64_t>(c.grid) ? t : c.grid);
 }
 
 // Largest n of the 1D entry points: the dense side is a tensor of 128-byte rows (n/32
@@ -126,14 +160,7 @@ int launch_minmax(const void *d_in, uint64_t n, double lambda, void *d_out, cuda
     const uint64_t nchunks = n * sizeof(T) / MM_CHUNK;
     if (nchunks >= static_cast<uint64_t>(sms)) {  // bulk-TMA streaming, 2 CTAs per SM
         constexpr int smem = MM_STAGES * MM_CHUNK;
-        static std::once_flag once;
-        static int attr_rc = CSZP2_OK;
-        std::call_once(once, [] {
-            if (cudaFuncSetAttribute(minmax_kernel_tma<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     smem) != cudaSuccess)
-                attr_rc = CSZP2_ERR_CUDA;
-        });
-        if (attr_rc != CSZP2_OK) return attr_rc;
+        if (int rc = set_smem(minmax_kernel_tma<T>, smem)) return rc;
         const uint64_t want = 2ull * sms;
         const int grid = static_cast<int>(nchunks < want ? nchunks : want);
         minmax_kernel_tma<T><<<grid, 256, smem, st>>>(static_cast<const T *>(d_in), n, lambda,
@@ -151,15 +178,15 @@ int launch_minmax(const void *d_in, uint64_t n, double lambda, void *d_out, cuda
 template <typename T, bool OUTLIER, int LOAD>
 int launch_compress_l(const void *d_in, const Geom &g, double eb, int eb_mode, int enc_mode,
                       void *d_out, uint64_t *d_out_bytes, cudaStream_t st, unsigned flags) {
-    static std::once_flag once;
-    static int attr_rc = CSZP2_OK;
-    static int grid_cache = 0;
     constexpr int smem = compress_smem_bytes<T>();
-    std::call_once(once, [] { attr_rc = set_smem(compress_kernel<T, OUTLIER, LOAD>, smem); });
-    if (attr_rc) return attr_rc;
-    const unsigned grid =
-        persistent_grid(compress_kernel<T, OUTLIER, LOAD>, NT_COMP, smem, g.T, &grid_cache);
+    if (int rc = set_smem(compress_kernel<T, OUTLIER, LOAD>, smem)) return rc;
+    const unsigned grid = persistent_grid(compress_kernel<T, OUTLIER, LOAD>, NT_COMP, smem, g.T);
     unsigned *ticket = reinterpret_cast<unsigned *>(static_cast<uint8_t *>(d_out) + stream_bound(g));
+    // the lookback descriptors (= the tile index, and its pad to O) and the tile ticket
+    // start from zero on every encode, so encode can be repeated on one buffer
+    // (FORMAT.md §2); skipped when the caller vouches that a prepare zeroed them
+    if (!(flags & CSZP2_FLAG_PREPARED))
+        if (int rc = zero_scratch(d_out, 64, g.O, g, st)) return rc;
     CUtensorMap map;
     int rc = make_tmap(&map, d_in, Traits<T>::DTYPE, g.nfull);
     if (rc) return rc;
@@ -188,13 +215,9 @@ int launch_compress(const void *d_in, const Geom &g, double eb, int eb_mode, int
 template <typename T>
 int launch_decompress(const void *d_cmp, void *d_out, const Geom &g, int *d_status,
                       cudaStream_t st) {
-    static std::once_flag once;
-    static int attr_rc = CSZP2_OK;
-    static int grid_cache = 0;
     constexpr int smem = decompress_smem_bytes<T>();
-    std::call_once(once, [] { attr_rc = set_smem(decompress_kernel<T>, smem); });
-    if (attr_rc) return attr_rc;
-    const unsigned grid = persistent_grid(decompress_kernel<T>, NT, smem, g.T, &grid_cache);
+    if (int rc = set_smem(decompress_kernel<T>, smem)) return rc;
+    const unsigned grid = persistent_grid(decompress_kernel<T>, NT, smem, g.T);
     CUtensorMap map;
     int rc = make_tmap(&map, d_out, Traits<T>::DTYPE, g.nfull);
     if (rc) return rc;
@@ -215,9 +238,8 @@ int geometry_nd(uint64_t nx, uint64_t ny, uint64_t nz, int ndim, GeomND *g) {
     g->nx = nx;
     g->ny = ny;
     g->nz = nz;
-    // n <= 2^40 (as 1D); checked without overflow
-    if (nx && ny && nz && (nx * ny > (1ull << 40) || nx * ny * nz / nz != nx * ny ||
-                           nx * ny * nz > (1ull << 40)))
+    // n <= MAX_N = 2^35 for compression and decompression alike; checked without overflow
+    if (nx && ny && nz && (nx * ny > MAX_N || nx * ny * nz / nz != nx * ny || nx * ny * nz > MAX_N))
         return CSZP2_ERR_ARG;
     g->n = nx * ny * nz;
     g->nbx = (nx + b - 1) / b;
@@ -234,12 +256,8 @@ uint64_t stream_bound_nd(const GeomND &g) { return roundup16(g.D + static_cast<u
 template <typename T, int NDIM, bool OUTLIER>
 int launch_compress_nd(const void *d_in, const GeomND &g, double eb, int eb_mode, int enc_mode,
                        void *d_out, uint64_t *d_out_bytes, cudaStream_t st) {
-    static std::once_flag once;
-    static int attr_rc = CSZP2_OK;
-    static int grid_cache = 0;
     constexpr int smem = ND_RING + 64;
-    std::call_once(once, [] { attr_rc = set_smem(compress_nd_kernel<T, NDIM, OUTLIER>, smem); });
-    if (attr_rc) return attr_rc;
+    if (int rc = set_smem(compress_nd_kernel<T, NDIM, OUTLIER>, smem)) return rc;
     unsigned *ticket = reinterpret_cast<unsigned *>(static_cast<uint8_t *>(d_out) + stream_bound_nd(g));
     HdrStatic hs;
     hs.word1 = 1u | (static_cast<uint32_t>(Traits<T>::DTYPE) << 8) |
@@ -247,7 +265,7 @@ int launch_compress_nd(const void *d_in, const GeomND &g, double eb, int eb_mode
     hs.eb_mode = static_cast<uint32_t>(eb_mode);
     hs.eb_user = eb;
     hs.flags = 0;
-    const unsigned grid = persistent_grid(compress_nd_kernel<T, NDIM, OUTLIER>, NT, smem, g.T, &grid_cache);
+    const unsigned grid = persistent_grid(compress_nd_kernel<T, NDIM, OUTLIER>, NT, smem, g.T);
     compress_nd_kernel<T, NDIM, OUTLIER><<<grid, NT, smem, st>>>(
         static_cast<const T *>(d_in), g, eb, eb_mode == CSZP2_EB_REL ? 1 : 0,
         static_cast<uint8_t *>(d_out), ticket, d_out_bytes, hs);
@@ -257,11 +275,8 @@ int launch_compress_nd(const void *d_in, const GeomND &g, double eb, int eb_mode
 template <typename T, int NDIM>
 int launch_decompress_nd(const void *d_cmp, void *d_out, const GeomND &g, int *d_status,
                          cudaStream_t st) {
-    static std::once_flag once;
-    static int attr_rc = CSZP2_OK;
     constexpr int smem = ND_STAGE + 64;
-    std::call_once(once, [] { attr_rc = set_smem(decompress_nd_kernel<T, NDIM>, smem); });
-    if (attr_rc) return attr_rc;
+    if (int rc = set_smem(decompress_nd_kernel<T, NDIM>, smem)) return rc;
     const unsigned grid = static_cast<unsigned>(g.T ? g.T : 1);
     decompress_nd_kernel<T, NDIM><<<grid, NT, smem, st>>>(static_cast<const uint8_t *>(d_cmp),
                                                           static_cast<T *>(d_out), g, d_status);
@@ -301,10 +316,9 @@ int cszp2_compress_prepare(const void *d_in, uint64_t n, int dtype, double eb, i
                            void *d_out, void *stream) {
     int rc = check_compress_args(d_in, n, dtype, eb, eb_mode, d_out);
     if (rc) return rc;
-    Geom g = geometry(n);
-    if (cudaMemsetAsync(d_out, 0, g.O, S(stream)) != cudaSuccess ||
-        cudaMemsetAsync(static_cast<uint8_t *>(d_out) + stream_bound(g), 0, 16, S(stream)) != cudaSuccess)
-        return CSZP2_ERR_CUDA;
+    // the header (REL's reduction scratch and eb_abs), the tile index and the ticket:
+    // one launch, so that cszp2_compress's encode needs none (CSZP2_FLAG_PREPARED)
+    if (int zr = zero_scratch(d_out, 0, geometry(n).O, geometry(n), S(stream))) return zr;
     if (eb_mode == CSZP2_EB_REL)
         return dtype == CSZP2_F32 ? launch_minmax<float>(d_in, n, eb, d_out, S(stream))
                                   : launch_minmax<double>(d_in, n, eb, d_out, S(stream));
@@ -325,10 +339,7 @@ int cszp2_compress_prepare_range(const void *d_in, uint64_t n, int dtype, double
     int rc = check_compress_args(d_in, n, dtype, eb, CSZP2_EB_REL, d_out);
     if (rc) return rc;
     if (!d_range || !aligned16(d_range)) return CSZP2_ERR_ARG;
-    Geom g = geometry(n);
-    if (cudaMemsetAsync(d_out, 0, g.O, S(stream)) != cudaSuccess ||
-        cudaMemsetAsync(static_cast<uint8_t *>(d_out) + stream_bound(g), 0, 16, S(stream)) != cudaSuccess)
-        return CSZP2_ERR_CUDA;
+    if (int zr = zero_scratch(d_out, 0, geometry(n).O, geometry(n), S(stream))) return zr;
     eb_from_range_kernel<<<1, 1, 0, S(stream)>>>(d_range, eb, static_cast<uint8_t *>(d_out));
     return launch_status();
 }
@@ -339,7 +350,8 @@ int cszp2_compress_encode_ex(const void *d_in, uint64_t n, int dtype, double eb,
     int rc = check_compress_args(d_in, n, dtype, eb, eb_mode, d_out);
     if (rc) return rc;
     if (enc_mode != CSZP2_ENC_PLAIN && enc_mode != CSZP2_ENC_OUTLIER) return CSZP2_ERR_ARG;
-    if (flags & ~(CSZP2_FLAG_CHAINED_SCAN | CSZP2_FLAG_LOAD_VEC | CSZP2_FLAG_LOAD_SCALAR)) return CSZP2_ERR_ARG;
+    if (flags & ~(CSZP2_FLAG_CHAINED_SCAN | CSZP2_FLAG_LOAD_VEC | CSZP2_FLAG_LOAD_SCALAR | CSZP2_FLAG_PREPARED))
+        return CSZP2_ERR_ARG;
     if ((flags & CSZP2_FLAG_LOAD_VEC) && (flags & CSZP2_FLAG_LOAD_SCALAR)) return CSZP2_ERR_ARG;
     Geom g = geometry(n);
     cudaStream_t st = S(stream);
@@ -363,7 +375,8 @@ int cszp2_compress(const void *d_in, uint64_t n, int dtype, double eb, int eb_mo
     if (enc_mode != CSZP2_ENC_PLAIN && enc_mode != CSZP2_ENC_OUTLIER) return CSZP2_ERR_ARG;
     int rc = cszp2_compress_prepare(d_in, n, dtype, eb, eb_mode, d_out, stream);
     if (rc) return rc;
-    return cszp2_compress_encode(d_in, n, dtype, eb, eb_mode, enc_mode, d_out, d_out_bytes, stream);
+    return cszp2_compress_encode_ex(d_in, n, dtype, eb, eb_mode, enc_mode, d_out, d_out_bytes, CSZP2_FLAG_PREPARED,
+                                    stream);
 }
 
 int cszp2_decompress(const void *d_cmp, void *d_out, uint64_t n, int dtype, int *d_status,

@@ -246,6 +246,7 @@ __device__ __forceinline__ uint32_t ld_u32_unaligned(const uint8_t *base, uint32
 // s >= R reduce to merges A[i] |= A[i+s] << s (rows [s, 2s) become zero) and the
 // remaining ones touch rows [0, R) only. Cost per 32 values: R=1: 31 ops, 2: 35,
 // 4: 48, 8: 84, 16: 176, 32: 400 — against 64 per plane for a bit-serial pack.
+// (Byte permutes (PRMT) for the S = 16 / 8 stages measured -1% on both kernels.)
 __host__ __device__ constexpr uint32_t stage_mask(int s) {
     return s == 16 ? 0x0000FFFFu
                    : (s == 8 ? 0x00FF00FFu : (s == 4 ? 0x0F0F0F0Fu : (s == 2 ? 0x33333333u : 0x55555555u)));
@@ -813,10 +814,19 @@ constexpr int RESOLVE_WARP = NT / 32;  // warp 8
 constexpr int NQ = 16;                 // queue slots (tiles staged ahead of the resolver)
 constexpr uint32_t BAR_PROD = 1;
 
+// The staging ring lives in a virtual byte space of RING_V per lap (a power of 2, so
+// u32 cursors wrap consistently) of which the first RING bytes exist: an allocation
+// never straddles RING (it moves to the next lap instead), so virtual position p is
+// physical byte p % RING_V and the room test is pos + bytes <= tail + RING_V.
+// 40 KiB: the most that keeps three f32 CTAs per SM (3 x (32 KiB tile + 40 KiB ring +
+// alignment + static) <= 228 KiB; f64: two CTAs with 64 KiB tiles); at CR ~2.5 a tile
+// stages ~14 KiB and stays in the ring for one lookback latency (~6 us at cfg4a), so
+// the 32 KiB ring of round 1 held only two of them.
 template <typename T>
 struct CompLayout {
     static constexpr uint32_t IN_BYTES = Traits<T>::TILE_BYTES;  // one TMA tile
-    static constexpr uint32_t RING = 32768;  // = the largest tile payload (256 x 128 B); a power of 2
+    static constexpr uint32_t RING = 40960;  // >= the largest tile payload (256 x 128 B)
+    static constexpr uint32_t RING_V = 65536;
     static constexpr int SMEM = IN_BYTES + RING + 64 + 1024;
 };
 template <typename T>
@@ -880,9 +890,10 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
     __shared__ uint32_t s_qagg[NQ], s_qpos[NQ];
     __shared__ uint8_t s_qbad[NQ];
     __shared__ uint32_t s_warp[2][NT / 32];  // tile_scan_1bar, by tile parity
+    __shared__ uint32_t s_tailb[2];          // s_tail as thread 0 acquired it before the scan, by tile parity
+    __shared__ uint32_t s_tail;              // ring bytes released by the resolver
     __shared__ uint32_t s_tkin;
     __shared__ uint64_t s_rel;            // producer warps done reading the input buffer
-    __shared__ volatile uint32_t s_tail;  // ring bytes released by the resolver
     __shared__ volatile uint32_t s_end;   // queue index of the end marker
 
     const int tid = threadIdx.x;
@@ -924,7 +935,8 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
         }
     };
 
-    for (uint32_t c = tid; c < LY::RING / 16; c += NT_COMP)  // staging ring starts zeroed
+    constexpr uint32_t RING = LY::RING, RING_V = LY::RING_V;
+    for (uint32_t c = tid; c < RING / 16; c += NT_COMP)  // staging ring starts zeroed
         reinterpret_cast<uint4 *>(ring)[c] = make_uint4(0, 0, 0, 0);
     if (tid == 0) {
         s_end = 0xFFFFFFFFu;
@@ -945,22 +957,36 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
         const auto K = make_consts(eb_abs, static_cast<T *>(nullptr));
         // ring allocation cursor and latest payload size: identical in every producer thread
         uint32_t head = 0, last_agg = 0;
+        // where a payload of `bytes` would go, and whether it fits now
+        auto place = [&](uint32_t bytes) {
+            uint32_t pos = (head + 15u) & ~15u;
+            if ((pos % RING_V) + bytes > RING) pos = (pos / RING_V + 1) * RING_V;
+            return pos;
+        };
+        auto fits = [&](uint32_t pos, uint32_t bytes, uint32_t tl) { return pos + bytes <= tl + RING_V || tl == head; };
         for (uint32_t it = 0;; ++it) {
             const int q = it % NQ;
-            // thread 0 takes the next ticket while the data is in flight (if the ring
-            // clearly has room for two more payloads); the atomic's result stays in a
-            // register until the buffer is released, so nothing waits on its round trip
+            // thread 0 takes the next ticket while the data is in flight if this tile's
+            // payload (estimated from the last one) fits in the ring now, i.e. its staging
+            // will not wait on a lookback while the ticket is held unpublished; the
+            // atomic's result stays in a register until the buffer is released, so
+            // nothing waits on its round trip
             uint32_t tk_next = 0;
             bool ahead = false;
             if (tid == 0) {
-                ahead = head - s_tail + 2 * last_agg + 64 <= LY::RING;
+                // the ring's free cursor, acquired: the resolver's clears of the freed bytes
+                // happen-before it, and the scan barrier hands it to every producer
+                const uint32_t tl = ld_acquire_cta(&s_tail);
+                s_tailb[it & 1] = tl;
+                const uint32_t est = min(BPT * 4u * L, last_agg + last_agg / 4u + 256u);
+                ahead = fits(place(est), est, tl);
                 if (ahead) tk_next = atomicAdd(ticket, 1u);
             }
             mbar_wait(&s_full, it & 1);
             const uint64_t t = s_tkin;  // published before the arrival we just waited for
             if (t >= T_eff) {           // end marker for the resolver (one arrival per warp)
                 if ((tid & 31) == 0) {
-                    if (it >= NQ) mbar_wait(&s_done[q], (it / NQ - 1) & 1);
+                    if (it >= NQ) mbar_wait(&s_done[q], (it / NQ - 1) & 1);  // slot free
                     if (tid == 0) s_end = it;
                     mbar_arrive(&s_staged[q]);
                 }
@@ -1073,9 +1099,11 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
             // thread from (head, agg); each waits for room itself. An empty ring always has
             // room (a payload that had to skip the ring's end can then never find the
             // skipped bytes still "in use").
-            uint32_t pos = (head + 15u) & ~15u;
-            if ((pos % LY::RING) + agg > LY::RING) pos = (pos / LY::RING + 1) * LY::RING;
-            while (pos + agg > s_tail + LY::RING && s_tail != head) __nanosleep(64);
+            // room with thread 0's acquired free cursor (bar.sync orders that acquire before
+            // every producer's staging stores); else each thread spins with acquire loads
+            const uint32_t pos = place(agg);
+            if (!fits(pos, agg, s_tailb[it & 1]))
+                while (!fits(pos, agg, ld_acquire_cta(&s_tail))) __nanosleep(64);
             head = pos + agg;
             last_agg = agg;
             if (active) out[g.O + b] = static_cast<uint8_t>(obyte);  // ❹ offset bytes
@@ -1083,7 +1111,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
             // ❷ payload staged in the ring at its tile-relative byte offset; bit planes
             // by an in-register transpose sized to the warp's largest fixed length
             {
-                const uint32_t st = (pos % LY::RING) + my_excl;
+                const uint32_t st = (pos % RING_V) + my_excl;
                 const uint32_t outl = a[0];
                 if (OUTLIER && nob) a[0] = 0;  // the outlier slot of every plane is 0
                 const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, static_cast<unsigned>(size ? fl : 0)));
@@ -1127,14 +1155,17 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
                 }
                 mbar_arrive(&s_staged[q]);
             }
-            if (tid == 0 && !ahead) {  // claim now, nothing unpublished held: wait for ring room first
-                while (head - s_tail + 2 * last_agg + 64 > LY::RING && head != s_tail) __nanosleep(64);
-                claim(atomicAdd(ticket, 1u));
-            }
+            // claim now: nothing unpublished is held, and the claimed tile publishes its
+            // aggregate before it can wait for ring room, so no wait is needed here
+            if (tid == 0 && !ahead) claim(atomicAdd(ticket, 1u));
         }
     } else {
         // ============================== resolver: ❸ then ❹, in tile order
+        // (Issuing the next queued tile's lookback window before this tile's copy was
+        // measured 5-13% slower: the early snapshot holds Waiting descriptors that have
+        // published by the time it is read, and every one costs a back-off re-poll.)
         const int lane = tid & 31;
+        const bool chained = (hs.flags & 1u) != 0;
         for (uint32_t it = 0;; ++it) {
             const int q = it % NQ;
             mbar_wait_backoff(&s_staged[q], (it / NQ) & 1, 100);
@@ -1146,7 +1177,6 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
             if (lane == 0) TRACE(t, 6, gtimer());
             bool rng = bad;
             uint64_t excl = 0;
-            const bool chained = (hs.flags & 1u) != 0;
             if (lane == 0) TRACE(t, 8, gtimer());
             if (g.T && t > 0) {
                 if (chained)  // ablation: plain chained scan (Fig 12 left)
@@ -1156,7 +1186,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
             }
             if (lane == 0) TRACE(t, 3, gtimer());
             const uint64_t dst0 = g.D + excl;
-            write_payload(ring + (pos % LY::RING), out, dst0, agg, lane, 32);
+            write_payload(ring + (pos % RING_V), out, dst0, agg, lane, 32);
             if (lane == 0) TRACE(t, 9, gtimer());
             if (t == T_eff - 1) {  // last tile: pads, header, d_out_bytes
                 const uint64_t dst1 = dst0 + agg;
@@ -1186,13 +1216,13 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
             }
             __syncwarp();  // every lane is done reading these ring bytes: clear them for reuse
             {
-                uint4 *z = reinterpret_cast<uint4 *>(ring + (pos % LY::RING));
+                uint4 *z = reinterpret_cast<uint4 *>(ring + (pos % RING_V));
                 for (uint32_t c = lane; c < (agg + 15u) / 16u; c += 32) z[c] = make_uint4(0, 0, 0, 0);
             }
-            __syncwarp();
+            __syncwarp();  // every lane's zero stores are ordered before lane 0's release below
             if (lane == 0) {
-                __threadfence_block();  // the zeros land before the producers may reuse the bytes
-                s_tail = pos + agg;     // in order, so the ring frees in order
+                __threadfence_block();  // release pattern: fence, then the relaxed cursor store
+                st_relaxed_cta(&s_tail, pos + agg);  // in order, so the ring frees in order
                 mbar_arrive(&s_done[q]);
             }
         }
@@ -1653,6 +1683,16 @@ __global__ void __launch_bounds__(NT) decompress_tilewise_kernel(const uint8_t *
         for (int i = 0; i < L; i++)
             if (b * L + i < g.n) out[b * L + i] = x[i];
     }
+}
+
+// ------------------------------------------------------------------ encode scratch
+// Zero `words` u64 from `p` (the header and/or the tile index = the lookback
+// descriptors, FORMAT.md §2) and the 16-byte tile ticket, in one launch.
+__global__ void zero_scratch_kernel(uint64_t *__restrict__ p, uint64_t words, uint4 *__restrict__ ticket) {
+    const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
+    for (uint64_t i = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x; i < words; i += stride)
+        p[i] = 0;
+    if (blockIdx.x == 0 && threadIdx.x == 0) *ticket = make_uint4(0, 0, 0, 0);
 }
 
 // ------------------------------------------------------------------ container index

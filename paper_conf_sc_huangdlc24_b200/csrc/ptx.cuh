@@ -34,6 +34,34 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t *bar, uint32_t parity) {
         : "memory");
     return ok != 0;
 }
+// Non-blocking test of a phase (never suspends the thread).
+__device__ __forceinline__ bool mbar_test(uint64_t *bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+    return ok != 0;
+}
+// CTA-scope acquire / relaxed accesses of a shared-memory word (the staging ring's free
+// cursor: with the resolver's fence before its relaxed store, the resolver's zero stores
+// happen-before a producer's reuse of the bytes).
+__device__ __forceinline__ uint32_t ld_acquire_cta(const uint32_t *p) {
+    uint32_t v;
+    asm volatile("ld.acquire.cta.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint32_t ld_relaxed_cta(const uint32_t *p) {
+    uint32_t v;
+    asm volatile("ld.relaxed.cta.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_relaxed_cta(uint32_t *p, uint32_t v) {
+    asm volatile("st.relaxed.cta.shared::cta.u32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
+}
 // Blocking wait: try_wait with a suspend-time hint, so a waiting warp sleeps in
 // hardware until the phase flips instead of spinning on issue slots.
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {

@@ -62,22 +62,26 @@ def compress_slab(x_slab: torch.Tensor, eb: float, eb_mode: str, enc_mode: str, 
 
     if rel_scope not in ("rank", "global"):
         raise ValueError("rel_scope must be 'rank' or 'global'")
-    if eb_mode == "rel" and rel_scope == "global":
-        x = x_slab.contiguous().view(-1)
-        if out is None:
-            out = torch.empty(compress_bound(x.numel(), x.dtype), dtype=torch.uint8, device=x.device)
-        if nbytes is None:
-            nbytes = torch.zeros(1, dtype=torch.int64, device=x.device)
-        cur = torch.cuda.current_stream() if stream is None else stream
-        with torch.cuda.stream(cur):  # the collective runs on the stream the kernels use
+    x = x_slab.contiguous().view(-1)
+    cur = torch.cuda.current_stream(x.device) if stream is None else stream
+    # every launch AND both collectives are ordered on `cur`: torch.distributed orders a
+    # collective after the current stream's work and the current stream after the
+    # collective, so the size all-gather reads d_out_bytes after the compressor wrote it
+    # and the container-index kernel reads the sizes after NCCL delivered them
+    with torch.cuda.device(x.device), torch.cuda.stream(cur):
+        if eb_mode == "rel" and rel_scope == "global":
+            if out is None:
+                out = torch.empty(compress_bound(x.numel(), x.dtype), dtype=torch.uint8, device=x.device)
+            if nbytes is None:
+                nbytes = torch.zeros(1, dtype=torch.int64, device=x.device)
             rng = reduce_range(value_range(x, stream=cur), group)
             compress_prepare_range(x, eb, rng, out, stream=cur)
-            compress_encode(x, eb, "rel", enc_mode, out, nbytes, stream=cur)
-    else:
-        out, nbytes = compress(x_slab, eb, eb_mode, enc_mode, out=out, out_bytes=nbytes, stream=stream)
-    if dist.is_available() and dist.is_initialized():
-        sizes = gather_sizes(nbytes, group)
-    else:
-        sizes = nbytes.view(1)
-    offsets = container_index(sizes, stream=stream)
+            compress_encode(x, eb, "rel", enc_mode, out, nbytes, stream=cur, prepared=True)
+        else:
+            out, nbytes = compress(x, eb, eb_mode, enc_mode, out=out, out_bytes=nbytes, stream=cur)
+        if dist.is_available() and dist.is_initialized():
+            sizes = gather_sizes(nbytes, group)
+        else:
+            sizes = nbytes.view(1)
+        offsets = container_index(sizes, stream=cur)
     return out, nbytes, offsets

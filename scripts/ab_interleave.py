@@ -26,6 +26,7 @@ def load(path):
     L.cszp2_compress_bound.argtypes = [u64, i32]
     L.cszp2_compress_prepare.argtypes = [vp, u64, i32, dbl, i32, vp, vp]
     L.cszp2_compress_encode.argtypes = [vp, u64, i32, dbl, i32, i32, vp, vp, vp]
+    L.cszp2_compress_encode_ex.argtypes = [vp, u64, i32, dbl, i32, i32, vp, vp, ctypes.c_uint, vp]
     L.cszp2_decompress.argtypes = [vp, vp, u64, i32, vp, vp]
     return L
 
@@ -61,8 +62,12 @@ def main():
                     L.cszp2_compress_prepare(vp(x.data_ptr()), n, dt, lam, ebm, vp(out.data_ptr()), sp)
                     e0, e1, e2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
                     e0.record(st)
-                    L.cszp2_compress_encode(vp(x.data_ptr()), n, dt, lam, ebm, enc, vp(out.data_ptr()),
-                                            vp(nb.data_ptr()), sp)
+                    # the kernel alone (FLAG_PREPARED: prepare zeroed the index); builds that
+                    # predate the flag reject it (ARG) and zero the index in prepare anyway
+                    if L.cszp2_compress_encode_ex(vp(x.data_ptr()), n, dt, lam, ebm, enc, vp(out.data_ptr()),
+                                                  vp(nb.data_ptr()), 8, sp) == 1:
+                        L.cszp2_compress_encode(vp(x.data_ptr()), n, dt, lam, ebm, enc, vp(out.data_ptr()),
+                                                vp(nb.data_ptr()), sp)
                     e1.record(st)
                     L.cszp2_decompress(vp(out.data_ptr()), vp(y.data_ptr()), n, dt, None, sp)
                     e2.record(st)

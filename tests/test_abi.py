@@ -53,5 +53,25 @@ def test_cpu_tensors_are_rejected():
 
     import paper_conf_sc_huangdlc24_b200 as cz
 
-    with pytest.raises(ValueError):
-        cz.compress(torch.zeros(10), 1e-3)
+    x = torch.zeros(10)
+    buf = torch.zeros(cz.compress_bound(10), dtype=torch.uint8)
+    nb = torch.zeros(1, dtype=torch.int64)
+    calls = [
+        lambda: cz.compress(x, 1e-3),
+        lambda: cz.compress_prepare(x, 1e-3, "rel", buf),
+        lambda: cz.compress_encode(x, 1e-3, "rel", "outlier", buf, nb),
+        lambda: cz.compress_encode_ex(x, 1e-3, "abs", "plain", buf, nb, flags=1),
+        lambda: cz.compress_prepare_range(x, 1e-3, torch.zeros(2, dtype=torch.float64), buf),
+        lambda: cz.value_range(x),
+        lambda: cz.decompress(buf, 10),
+        lambda: cz.decompress_range(buf, 10, 0, 5),
+        lambda: cz.decompress_tilewise(buf, 10),
+        lambda: cz.read_header(buf),
+        lambda: cz.container_index(nb),
+        lambda: cz.compress_nd(torch.zeros(4, 4), 1e-3),
+        lambda: cz.decompress_nd(buf, (4, 4)),
+        lambda: cz.compress_host(x, 1e-3, "abs", "plain", x, buf, buf),
+    ]
+    for i, c in enumerate(calls):
+        with pytest.raises(ValueError):
+            c()

@@ -438,7 +438,7 @@ def test_c_abi_rejects_invalid_arguments():
     assert L.cszp2_compress(p(x, 4), 10, 0, 1e-3, 0, 0, p(out), p(nb), s) == E       # misaligned in
     assert L.cszp2_compress(p(x), 10, 0, 1e-3, 0, 0, p(out, 8), p(nb), s) == E       # misaligned out
     assert L.cszp2_compress(p(x), (1 << 35) + 1, 0, 1e-3, 0, 0, p(out), p(nb), s) == E  # n too large
-    assert L.cszp2_compress_encode_ex(p(x), 10, 0, 1e-3, 0, 0, p(out), p(nb), 8, s) == E  # flags
+    assert L.cszp2_compress_encode_ex(p(x), 10, 0, 1e-3, 0, 0, p(out), p(nb), 16, s) == E  # flags
     assert L.cszp2_compress_encode_ex(p(x), 10, 0, 1e-3, 0, 0, p(out), p(nb), 6, s) == E  # vec+scalar
     assert L.cszp2_decompress(None, p(x), 10, 0, None, s) == E
     assert L.cszp2_decompress(p(out), p(x, 4), 10, 0, None, s) == E
@@ -464,3 +464,48 @@ def test_incompressible_many_tiles(dtype, enc):
     xh = (rng.standard_normal(n) * 1e3).astype(dtype)
     got = check_roundtrip(xh, 1e-5, "abs", enc)
     assert got is not None and got.size > 0.4 * xh.nbytes  # near-incompressible (f64: ~0.45)
+
+
+@pytest.mark.parametrize("eb_mode", ["abs", "rel"])
+def test_encode_repeated_on_one_buffer(eb_mode):
+    """cszp2_compress_encode re-zeroes its lookback descriptors and ticket, so encoding
+    again into the same d_out (after one prepare, or with another mode) gives the
+    oracle's stream every time (include/cszp2.h)."""
+    rng = np.random.default_rng(77)
+    xh = np.cumsum(rng.standard_normal(8192 * 30 + 45)).astype(np.float32)
+    x = torch.from_numpy(xh).to(DEV)
+    out = torch.full((cz.compress_bound(x.numel()),), 0xAA, dtype=torch.uint8, device=DEV)
+    nb = torch.zeros(1, dtype=torch.int64, device=DEV)
+    cz.compress_prepare(x, 1e-3, eb_mode, out)
+    for enc in ("outlier", "outlier", "plain", "outlier"):
+        cz.compress_encode(x, 1e-3, eb_mode, enc, out, nb)
+        torch.cuda.synchronize()
+        ref, rc = oracle.compress(xh, 1e-3, EBM[eb_mode], ENC[enc])
+        assert rc == oracle.OK and int(nb.item()) == ref.size
+        np.testing.assert_array_equal(out[:ref.size].cpu().numpy(), ref)
+
+
+def test_binding_validates_buffers():
+    """The ctypes binding refuses buffers the kernels would overrun or misread
+    (ADVICE r1): short / wrongly typed stream buffers, output tensors of the wrong
+    length, dtype or layout, status / size words of the wrong type."""
+    x = torch.randn(10000, device=DEV)
+    bound = cz.compress_bound(x.numel())
+    good = torch.empty(bound, dtype=torch.uint8, device=DEV)
+    nb = torch.zeros(1, dtype=torch.int64, device=DEV)
+    bad_calls = [
+        lambda: cz.compress(x, 1e-3, out=torch.empty(bound - 1, dtype=torch.uint8, device=DEV)),
+        lambda: cz.compress(x, 1e-3, out=torch.empty(bound // 4 + 1, dtype=torch.int32, device=DEV)),
+        lambda: cz.compress(x, 1e-3, out=good, out_bytes=torch.zeros(1, dtype=torch.int32, device=DEV)),
+        lambda: cz.compress(x.to(torch.float16), 1e-3),
+        lambda: cz.compress_encode(x[::2], 1e-3, "abs", "plain", good, nb),
+        lambda: cz.compress_prepare(x, 1e-3, "rel", good[:100]),
+        lambda: cz.decompress(good, x.numel(), out=torch.empty(x.numel() - 1, device=DEV)),
+        lambda: cz.decompress(good, x.numel(), out=torch.empty(2 * x.numel(), device=DEV)[::2]),
+        lambda: cz.decompress(good, x.numel(), status=torch.zeros(1, dtype=torch.int64, device=DEV)),
+        lambda: cz.decompress_range(good, x.numel(), 0, 10, out=torch.empty(9, device=DEV)),
+        lambda: cz.container_index(nb, out=torch.empty(1, dtype=torch.int64, device=DEV)),
+    ]
+    for c in bad_calls:
+        with pytest.raises(ValueError):
+            c()

@@ -104,30 +104,38 @@ class _OracleCodec:
         import oracle
 
         s, rc = oracle.compress(x.numpy(), self.eb, self.eb_mode, self.enc)
-        assert rc == oracle.OK
+        assert rc in (oracle.OK, oracle.ERR_RANGE)  # a RANGE stream is still a stream
         buf = torch.zeros(oracle.compress_bound(x.numel()) + 16, dtype=torch.uint8)
         buf[: s.size] = torch.from_numpy(s)
         return buf, torch.tensor([s.size], dtype=torch.int64)
 
-    def decompress(self, cmp, n, out):
+    def decompress(self, cmp, n, out, status, stream=None):
         import oracle
 
         y, rc = oracle.decompress(cmp.numpy(), n, np.float32 if out.dtype == torch.float32 else np.float64)
-        assert rc == oracle.OK
-        out.copy_(torch.from_numpy(y))
+        status.fill_(rc)
+        if rc == oracle.OK:
+            out.copy_(torch.from_numpy(y))
 
 
-def _cag_worker(rank, world, port, n, eb, enc, result_q):
+def _cag_worker(rank, world, port, n, eb, enc, result_q, nan_rank=-1):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
+        from paper_conf_sc_huangdlc24_b200 import CszpError
         from paper_conf_sc_huangdlc24_b200.collective import compressed_all_gather
         from synthetic import make_field
 
         x = make_field("cfg2", "cpu", rank * n, n)  # shard r of one field
+        if rank == nan_rank:
+            x[n // 3] = float("nan")
         stats = {}
-        y = compressed_all_gather(x, eb, "rel", "outlier", codec=_OracleCodec(eb, 1, enc), stats=stats)
+        try:
+            y = compressed_all_gather(x, eb, "rel", "outlier", codec=_OracleCodec(eb, 1, enc), stats=stats)
+        except CszpError as e:
+            result_q.put((rank, "error", str(e)))
+            return
         result_q.put((rank, y.numpy().tobytes(), stats))
     finally:
         dist.destroy_process_group()
@@ -163,6 +171,24 @@ def test_compressed_all_gather_two_ranks(orc, enc):
         assert stats["sizes"] == sizes
         assert stats["slot"] == (max(sizes) + 15) // 16 * 16
         assert stats["wire_bytes"] == world * stats["slot"] < stats["raw_bytes"]
+
+
+def test_compressed_all_gather_reports_a_bad_shard(orc):
+    """A shard whose stream has RANGE status (a NaN, FORMAT.md §6.3) must not come back
+    as data: every rank raises CszpError naming that rank."""
+    world, n, eb = 2, 2 * 8192 + 32, 1e-4
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_cag_worker, args=(r, world, port, n, eb, 1, q, 1)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted([q.get(timeout=120) for _ in range(world)], key=lambda r: r[0])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for rank, kind, msg in res:
+        assert kind == "error" and "rank 1" in msg and "status 3" in msg
 
 
 def _grel_worker(rank, world, port, n, lam, enc, result_q):
