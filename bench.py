@@ -89,8 +89,9 @@ class ClockSampler:
          "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
          "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
 
-    def __init__(self, gpu_index: int):
+    def __init__(self, gpu_index: int, period_ms: int = 50):
         self.gpu = gpu_index
+        self.period_ms = period_ms
         self.proc = None
         self.raw = []
 
@@ -98,7 +99,7 @@ class ClockSampler:
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
-                 "-lms", "50"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+                 "-lms", str(self.period_ms)], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
             # nvidia-smi takes a few hundred ms to start: wait for its first sample, so
@@ -467,8 +468,13 @@ def main():
     # every other BASELINE config, N=1 only (configs 1-4 are single-GPU configs)
     sweep = None
     if world == 1 and not args.no_configs:
-        with ClockSampler(local) as sclk:
-            sweep = run_config_sweep(args, cz, dev, stream, peak, sclk)
+        with ClockSampler(local, period_ms=10) as sclk:
+            rows = run_config_sweep(args, cz, dev, stream, peak, sclk)
+        sweep = {"clocks": sclk.summary(), "entries": rows,
+                 "note": "per entry: kernel-only roofline fractions (algorithmic bytes = field + stream) and "
+                         "whole-direction GB/s (compress incl. the REL min/max pass), CUDA events on the "
+                         "launching stream, L2 flushed before every timed direction; clocks per entry are "
+                         "the nvidia-smi samples (10 ms) that fell inside it, the sweep's are above"}
 
     # cpu_baseline: the oracle as it stands, on a bounded sample, rank 0 at N=1 only
     cpu = cpu_mt = None
@@ -499,7 +505,10 @@ def main():
             "cpu_baseline_all_cores": cpu_mt,
             "e2e": e2e,
             "clocks": clocks,
-            "gpu_launches": args.steps * (3 + (1 if world > 1 else 0)),
+            # our kernels per step: prepare = zero_scratch (+ minmax for REL; global REL: minmax +
+            # zero_scratch + eb_from_range), compress, decompress (+ container index at N > 1)
+            "gpu_launches": args.steps * ((3 if glob else (2 if spec.eb_mode == "rel" else 1)) + 2
+                                          + (1 if world > 1 else 0)),
             "plain_mode": plain,
             "configs": sweep,
         }

@@ -105,13 +105,47 @@ __device__ __forceinline__ bool interior_vec(const GeomND &g, const BlockOrigin 
            o.z0 + S::BZ <= g.nz;
 }
 
-// one 32-bit word to smem at any byte position (neighbouring blocks own the other bytes)
-__device__ __forceinline__ void put_word(uint8_t *base, uint32_t pos, uint32_t w) {
-    if ((pos & 3u) == 0) {
-        *reinterpret_cast<uint32_t *>(base + pos) = w;
-    } else {
-        for (int j = 0; j < 4; j++) base[pos + j] = static_cast<uint8_t>(w >> (8 * j));
+// One block's nD payload (FORMAT.md §7: sign 8 B, nob outlier bytes, then planes
+// k = 0..fl-1 as (lo word, hi word)) to smem at byte `st` (any alignment). With the
+// plane region at ps = st + 8 + nob, r = ps & 3 and P_k the k-th plane word
+// (P_2j = lo[j], P_2j+1 = hi[j]; P_-1, P_-2, P_-3 the header words ending at ps), the
+// aligned word at ps - r + 4k is funnel(P_k-1, P_k, 8r): every aligned word that lies
+// inside the payload is one 32-bit store; the <= 3 head bytes and <= 3 tail bytes, whose
+// words the neighbouring blocks share, are byte stores. No atomics and no pre-zeroed
+// memory (each byte of the ring has exactly one writer).
+template <int R>
+__device__ __forceinline__ void stage_payload_nd(uint8_t *base, uint32_t st, uint64_t sign, uint32_t outl, int nob,
+                                                 int fl, const uint32_t (&lo)[32], const uint32_t (&hi)[32]) {
+    const uint32_t h0 = static_cast<uint32_t>(sign), h1 = static_cast<uint32_t>(sign >> 32), h2 = outl;
+    const uint32_t ps = st + 8u + nob;
+    const uint32_t r = ps & 3u;
+    const uint32_t sh = 8u * r;
+    uint32_t *w = reinterpret_cast<uint32_t *>(base + ps - r);
+    const uint32_t pm1 = static_cast<uint32_t>(((static_cast<uint64_t>(h2) << 32) | h1) >> (8 * nob));  // [4+nob, 8+nob)
+    const uint32_t pm2 = static_cast<uint32_t>(sign >> (8 * nob));                                   // [nob, nob+4)
+    const uint32_t pm3 = static_cast<uint32_t>(static_cast<uint64_t>(h0) << (32 - 8 * nob));  // top nob bytes
+    w[-1] = __funnelshift_l(pm2, pm1, sh);  // payload bytes [4 + nob - r, 8 + nob - r): always inside
+    if (static_cast<uint32_t>(nob) >= r) w[-2] = __funnelshift_l(pm3, pm2, sh);
+    if (nob == 4 && r == 0) w[-3] = h0;
+    // head bytes [0, hb): the payload bytes before the first word written above
+    const uint32_t hb = (nob == 4 && r == 0) ? 0u : (static_cast<uint32_t>(nob) >= r ? nob - r : 4u + nob - r);
+#pragma unroll
+    for (uint32_t i = 0; i < 3; i++)
+        if (i < hb) base[st + i] = static_cast<uint8_t>(h0 >> (8 * i));
+    uint32_t prev = pm1;
+#pragma unroll
+    for (int j = 0; j < R; j++) {
+        if (j < fl) {
+            w[2 * j] = __funnelshift_l(prev, lo[j], sh);
+            w[2 * j + 1] = __funnelshift_l(lo[j], hi[j], sh);
+            prev = hi[j];
+        }
     }
+    // tail bytes: the last r payload bytes (the top r bytes of the last word)
+    uint8_t *tb = base + ps - r + 8u * fl;
+#pragma unroll
+    for (uint32_t i = 0; i < 3; i++)
+        if (i < r) tb[i] = static_cast<uint8_t>(prev >> (8 * (4 - r + i)));
 }
 
 constexpr uint32_t ND_STAGE = BPT * 4 * LND + 64;  // max tile payload + slack (decompression)
@@ -137,8 +171,8 @@ __global__ void __launch_bounds__(NT, 2) compress_nd_kernel(const T *__restrict_
                                                             const HdrStatic hs) {
     extern __shared__ uint8_t stage_raw[];
     uint8_t *ring = smem_align<16>(stage_raw);
-    __shared__ uint32_t s_warp[NT / 32];
-    __shared__ uint32_t s_tk;
+    __shared__ uint32_t s_warp[2][NT / 32];  // tile_scan_1bar, by tile parity
+    __shared__ uint32_t s_tk[2];             // the claimed ticket of each iteration, by parity
     __shared__ uint64_t s_excl;
     __shared__ bool s_rng;
     const int tid = threadIdx.x;
@@ -157,8 +191,10 @@ __global__ void __launch_bounds__(NT, 2) compress_nd_kernel(const T *__restrict_
     LookbackWindow w;
 
     // resolve the deferred tile (warp 0: lookback; tile 0 / no index: 0), write its
-    // payload from the ring, and for the last tile the pads, header and d_out_bytes
-    auto flush_prev = [&]() {
+    // payload from the ring, and for the last tile the pads, header and d_out_bytes.
+    // claim_slot >= 0: thread 0 then claims the next tile into s_tk[claim_slot] — after
+    // the lookback, so a claimed tile never waits on one before it publishes.
+    auto flush_prev = [&](int claim_slot) {
         if (tid < 32) {
             bool rng = prev_bad;
             uint64_t e = 0;
@@ -166,9 +202,10 @@ __global__ void __launch_bounds__(NT, 2) compress_nd_kernel(const T *__restrict_
             if (tid == 0) {
                 s_excl = e;
                 s_rng = rng;
+                if (claim_slot >= 0) s_tk[claim_slot] = atomicAdd(ticket, 1u);
             }
         }
-        __syncthreads();  // s_excl visible; the ring bytes of the deferred tile are complete
+        __syncthreads();  // s_excl (and the ticket) visible; the deferred tile's ring bytes complete
         const uint64_t dst0 = g.D + s_excl;
         write_payload(ring + (prev_pos % ND_RING), out, dst0, prev_agg, tid, NT);
         if (prev_t == T_eff - 1) {  // last tile: pads, header, d_out_bytes
@@ -202,10 +239,10 @@ __global__ void __launch_bounds__(NT, 2) compress_nd_kernel(const T *__restrict_
         have_prev = false;
     };
 
-    for (;;) {
-        if (tid == 0) s_tk = atomicAdd(ticket, 1u);  // in-order tiles: forward progress
-        __syncthreads();
-        const uint64_t t = s_tk;
+    if (tid == 0) s_tk[0] = atomicAdd(ticket, 1u);  // in-order tiles: forward progress
+    __syncthreads();
+    for (uint32_t it = 0;; ++it) {
+        const uint64_t t = s_tk[it & 1];
         if (t >= T_eff) break;
 
         const uint64_t b = t * BPT + tid;
@@ -278,10 +315,11 @@ __global__ void __launch_bounds__(NT, 2) compress_nd_kernel(const T *__restrict_
         }
         if (!K.ok) bad = true;
 
-        // ---- ❸ intra-tile scan; publish the aggregate at once (never behind a lookback)
-        const bool any_bad = __syncthreads_or(bad);
+        // ---- ❸ intra-tile scan (one barrier, with the range flag); publish the
+        //      aggregate at once (never behind a lookback)
         uint32_t agg;
-        const uint32_t my_excl = cta_exclusive_scan(size, s_warp, &agg);
+        bool any_bad;
+        const uint32_t my_excl = tile_scan_1bar(size, bad, s_warp[it & 1], &agg, &any_bad, 0);
         if (tid == 0 && g.T) publish_aggregate(index, t, agg, any_bad);
         if (active) out[g.O + b] = static_cast<uint8_t>(obyte);
 
@@ -289,7 +327,7 @@ __global__ void __launch_bounds__(NT, 2) compress_nd_kernel(const T *__restrict_
         uint32_t pos = have_prev ? ((prev_pos + prev_agg + 15u) & ~15u) : 0u;
         if ((pos % ND_RING) + agg > ND_RING) pos = (pos / ND_RING + 1) * ND_RING;
         if (have_prev && pos + agg > prev_pos + ND_RING) {
-            flush_prev();
+            flush_prev(-1);
             pos = 0;
         }
 
@@ -317,24 +355,25 @@ __global__ void __launch_bounds__(NT, 2) compress_nd_kernel(const T *__restrict_
         }
         if (size) {
             uint8_t *stg = ring + (pos % ND_RING);
-            uint32_t p = my_excl;
-            put_word(stg, p, static_cast<uint32_t>(sign));
-            put_word(stg, p + 4, static_cast<uint32_t>(sign >> 32));
-            p += 8;
-            for (int j = 0; j < nob; j++) stg[p + j] = static_cast<uint8_t>(outl >> (8 * j));
-            p += nob;
-#pragma unroll
-            for (int k = 0; k < 32; k++) {
-                if (k < fl) {
-                    put_word(stg, p + 8 * k, lo[k]);
-                    put_word(stg, p + 8 * k + 4, hi[k]);
-                }
-            }
+            if (flw <= 4)
+                stage_payload_nd<4>(stg, my_excl, sign, outl, nob, fl, lo, hi);
+            else if (flw <= 8)
+                stage_payload_nd<8>(stg, my_excl, sign, outl, nob, fl, lo, hi);
+            else if (flw <= 16)
+                stage_payload_nd<16>(stg, my_excl, sign, outl, nob, fl, lo, hi);
+            else
+                stage_payload_nd<32>(stg, my_excl, sign, outl, nob, fl, lo, hi);
         }
 
         // ---- the deferred tile: its window has been in flight since last iteration
-        if (have_prev) flush_prev();  // (its first barrier also completes this tile's staging)
-        else __syncthreads();
+        //      (its first barrier also completes this tile's staging and hands out the
+        //      next ticket)
+        if (have_prev) {
+            flush_prev((it + 1) & 1);
+        } else {
+            if (tid == 0) s_tk[(it + 1) & 1] = atomicAdd(ticket, 1u);
+            __syncthreads();
+        }
 
         // ---- this tile becomes the deferred one; issue its lookback window now
         have_prev = true;
@@ -344,7 +383,7 @@ __global__ void __launch_bounds__(NT, 2) compress_nd_kernel(const T *__restrict_
         prev_bad = any_bad;
         if (tid < 32 && g.T && t > 0) lookback_issue(index, static_cast<int64_t>(t) - 1, w);
     }
-    if (have_prev) flush_prev();
+    if (have_prev) flush_prev(-1);
 }
 
 template <typename T, int NDIM>

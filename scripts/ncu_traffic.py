@@ -25,7 +25,7 @@ def capture(cfg, enc):
     from synthetic import CONFIGS
 
     per_round = "3" if CONFIGS[cfg].eb_mode == "rel" else "2"  # ABS has no min/max launch
-    rep = os.path.join(ROOT, "gpurun_out", f"traffic_{cfg}_{enc}")
+    rep = os.path.join("/tmp", f"traffic_{cfg}_{enc}")  # reports stay off gpurun_out (64 MiB cap)
     # prof_one: (prepare = memset + minmax, compress, decompress) x 3; skip the first round
     cmd = ["ncu", "--set", "full", "--clock-control", "none", "--kernel-name-base", "function",
            "-k", "regex:^(minmax_kernel|compress_kernel|decompress_kernel)", "-s", per_round, "-c", per_round,
@@ -39,7 +39,8 @@ def capture(cfg, enc):
     res = {}
     for r in data:
         name = r[hdr.index("Kernel Name")]
-        k = next((k for k in KERNELS if name.startswith(k)), None)
+        # demangled or base names: test the longer name first (it contains the shorter)
+        k = next((k for k in ("decompress_kernel", "compress_kernel", "minmax_kernel") if k in name), None)
         if k is None:
             continue
         f = lambda m: float(r[hdr.index(m)].replace(",", ""))  # noqa: E731
@@ -47,6 +48,7 @@ def capture(cfg, enc):
         res[f"{cfg}/{enc}/{k}"] = {"dram_bytes": rd + wr, "dram_read": rd, "dram_write": wr,
                                    "duration_ns": f("gpu__time_duration.sum"),
                                    "source": "ncu --set full --clock-control none, one launch (2nd round)"}
+    os.remove(rep + ".ncu-rep")
     return res
 
 
