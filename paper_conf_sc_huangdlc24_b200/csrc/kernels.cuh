@@ -6,12 +6,14 @@
 //                      one fused pass (Fig 4)
 //   decompress_kernel  ❸ (O(1) from the persisted tile index) → ❹ → ❷⁻¹ → ❶⁻¹
 //
-// B200 design: one CTA = one tile of 256 blocks (8192 f32 values);
-// one thread = one 32-value block (block-level data parallelism). Tiles move
-// between HBM and shared memory with TMA: 2D tensor maps with 128-byte swizzle for
-// the dense value side (so thread-per-block 16-byte shared accesses are
-// bank-conflict free), 1D bulk copies for the byte-granular compressed side.
-// Bit planes are packed/unpacked with add.cc/addc carry chains (2 ops per bit).
+// B200 design: persistent CTAs that claim tiles of 256 blocks (8192 f32
+// values) in order from an atomic ticket (compression) or walk tiles c, c+G, ...
+// (decompression); one thread = one 32-value block (block-level data parallelism,
+// P:176). Tiles move between HBM and shared memory with TMA: 2D tensor maps with
+// 128-byte swizzle for the dense value side (so thread-per-block 16-byte shared
+// accesses are bank-conflict free), 1D bulk copies for the byte-granular compressed
+// side. Bit planes are packed/unpacked by in-register 32x32 bit transposes sized to
+// the warp's largest fixed length.
 #pragma once
 #include <cstdint>
 #include <type_traits>
@@ -223,16 +225,6 @@ __device__ __forceinline__ void store_block(uint8_t *tile, uint32_t r, const dou
 }
 
 // ------------------------------------------------------------------ byte-granular smem access
-__device__ __forceinline__ void st_u32_unaligned(uint8_t *p, uint32_t w) {
-    if ((reinterpret_cast<uintptr_t>(p) & 3u) == 0) {
-        *reinterpret_cast<uint32_t *>(p) = w;
-    } else {
-        p[0] = static_cast<uint8_t>(w);
-        p[1] = static_cast<uint8_t>(w >> 8);
-        p[2] = static_cast<uint8_t>(w >> 16);
-        p[3] = static_cast<uint8_t>(w >> 24);
-    }
-}
 __device__ __forceinline__ uint32_t ld_u32_unaligned(const uint8_t *base, uint32_t pos) {
     const uint32_t *w = reinterpret_cast<const uint32_t *>(base + (pos & ~3u));
     return __funnelshift_r(w[0], w[1], 8u * (pos & 3u));
@@ -376,12 +368,6 @@ __device__ __forceinline__ void load_planes(const uint8_t *base, uint32_t pos, u
 }
 
 // ------------------------------------------------------------------ scans
-__device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-    return v;
-}
-
 // Exclusive scan of one u32 per thread over the NT threads 0..NT-1, synchronised
 // with barrier `bar_id` (0 = the whole CTA). Returns the exclusive prefix;
 // *total receives the sum. Contains two barriers.

@@ -2,9 +2,10 @@
 // §VI-D / Table VI: 2D Lorenzo on 8x8 blocks and 3D Lorenzo on 4x4x4
 // blocks (L = 64), same Plain/Outlier FLE, same decoupled-lookback concatenation
 // (FORMAT.md §7). The paper keeps them out of the main design because they cost
-// throughput (>50%); these kernels favour simplicity over speed: one CTA per
-// tile (dynamic ticket), one thread per 64-value block, values gathered straight
-// from global memory.
+// throughput (>50%). Compression: persistent CTAs claiming tiles in order from
+// an atomic ticket, one thread per 64-value block, values gathered straight from
+// global memory (16-byte rows), the lookback deferred by one tile. Decompression: one
+// CTA per tile, the payload located in O(1) by the tile index and bulk-loaded.
 #pragma once
 #include "kernels.cuh"
 

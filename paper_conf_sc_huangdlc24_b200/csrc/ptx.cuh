@@ -1,5 +1,6 @@
-// ptx.cuh — thin inline-PTX wrappers for sm_100a: mbarrier, TMA (tensor and
-// 1D bulk), proxy fences, acquire/release global accesses, carry-chain adds.
+// ptx.cuh — thin inline-PTX wrappers for sm_100a: mbarrier, named barriers, TMA
+// (tensor and 1D bulk), proxy fences, relaxed / acquire accesses for the lookback
+// descriptors and the staging ring's cursor.
 #pragma once
 #include <cstdint>
 #include <cuda.h>
@@ -34,29 +35,12 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t *bar, uint32_t parity) {
         : "memory");
     return ok != 0;
 }
-// Non-blocking test of a phase (never suspends the thread).
-__device__ __forceinline__ bool mbar_test(uint64_t *bar, uint32_t parity) {
-    uint32_t ok;
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t"
-        "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
-        "selp.u32 %0, 1, 0, p;\n\t}"
-        : "=r"(ok)
-        : "r"(smem_u32(bar)), "r"(parity)
-        : "memory");
-    return ok != 0;
-}
 // CTA-scope acquire / relaxed accesses of a shared-memory word (the staging ring's free
 // cursor: with the resolver's fence before its relaxed store, the resolver's zero stores
 // happen-before a producer's reuse of the bytes).
 __device__ __forceinline__ uint32_t ld_acquire_cta(const uint32_t *p) {
     uint32_t v;
     asm volatile("ld.acquire.cta.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
-    return v;
-}
-__device__ __forceinline__ uint32_t ld_relaxed_cta(const uint32_t *p) {
-    uint32_t v;
-    asm volatile("ld.relaxed.cta.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
     return v;
 }
 __device__ __forceinline__ void st_relaxed_cta(uint32_t *p, uint32_t v) {
@@ -86,17 +70,6 @@ __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
 __device__ __forceinline__ void named_sync(uint32_t id, uint32_t n) {
     asm volatile("barrier.cta.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
 }
-__device__ __forceinline__ bool named_sync_or(uint32_t id, uint32_t n, bool v) {
-    uint32_t r;
-    asm volatile(
-        "{\n\t.reg .pred p, q;\n\tsetp.ne.u32 p, %1, 0;\n\t"
-        "barrier.cta.red.or.pred q, %2, %3, p;\n\tselp.u32 %0, 1, 0, q;\n\t}"
-        : "=r"(r)
-        : "r"(static_cast<uint32_t>(v)), "r"(id), "r"(n)
-        : "memory");
-    return r != 0;
-}
-
 // Wait with a nanosleep back-off between polls: for warps whose wake-up latency
 // matters less than the issue slots their polling would take from busy warps.
 __device__ __forceinline__ void mbar_wait_backoff(uint64_t *bar, uint32_t parity, uint32_t ns) {
@@ -104,15 +77,6 @@ __device__ __forceinline__ void mbar_wait_backoff(uint64_t *bar, uint32_t parity
 }
 
 // ---------------------------------------------------------------- TMA
-// 2D tensor tile global -> shared (completes on an mbarrier).
-__device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, int x, int y,
-                                            uint64_t *bar) {
-    asm volatile(
-        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
-        " [%0], [%1, {%2, %3}], [%4];" ::"r"(smem_u32(dst)),
-        "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(smem_u32(bar))
-        : "memory");
-}
 // 2D tensor tile shared -> global (bulk group).
 __device__ __forceinline__ void tma_store_2d(const CUtensorMap *map, int x, int y,
                                              const void *src) {
@@ -157,19 +121,11 @@ __device__ __forceinline__ void bulk_load(void *dst, const void *src, uint32_t b
         "l"(src), "r"(bytes), "r"(smem_u32(bar))
         : "memory");
 }
-__device__ __forceinline__ void bulk_store(void *dst, const void *src, uint32_t bytes) {
-    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst),
-                 "r"(smem_u32(src)), "r"(bytes)
-                 : "memory");
-}
 __device__ __forceinline__ void bulk_commit() {
     asm volatile("cp.async.bulk.commit_group;" ::: "memory");
 }
 __device__ __forceinline__ void bulk_wait_read0() {
     asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
-}
-__device__ __forceinline__ void bulk_wait0() {
-    asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
 }
 // make generic-proxy shared-memory writes visible to the async (TMA) proxy
 __device__ __forceinline__ void fence_proxy_async_smem() {
@@ -177,11 +133,6 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
 }
 
 // ---------------------------------------------------------------- ordering
-__device__ __forceinline__ uint64_t ld_acquire_u64(const uint64_t *p) {
-    uint64_t v;
-    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-    return v;
-}
 // relaxed (but strong, gpu-scope) load: several can be in flight at once, unlike
 // ld.acquire which orders every later access behind itself
 __device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t *p) {
@@ -192,23 +143,4 @@ __device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t *p) {
 __device__ __forceinline__ void st_relaxed_u64(uint64_t *p, uint64_t v) {
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
-__device__ __forceinline__ void fence_acq_rel_gpu() {
-    asm volatile("fence.acq_rel.gpu;" ::: "memory");
-}
-__device__ __forceinline__ void st_release_u64(uint64_t *p, uint64_t v) {
-    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-__device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t *p) {
-    uint32_t v;
-    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-
-// ---------------------------------------------------------------- carry chains
-// b <- 2b (carry = old top bit of b); w <- 2w + carry. One plane bit moves from
-// value register b to plane word w (bit-plane pack, top plane first).
-__device__ __forceinline__ void shift_bit_into(uint32_t &b, uint32_t &w) {
-    asm("add.cc.u32 %0, %0, %0;\n\taddc.u32 %1, %1, %1;" : "+r"(b), "+r"(w));
-}
-
 }  // namespace cszp2
