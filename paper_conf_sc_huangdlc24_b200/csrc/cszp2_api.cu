@@ -265,8 +265,8 @@ int launch_compress_nd(const void *d_in, const GeomND &g, double eb, int eb_mode
     hs.eb_mode = static_cast<uint32_t>(eb_mode);
     hs.eb_user = eb;
     hs.flags = 0;
-    const unsigned grid = persistent_grid(compress_nd_kernel<T, NDIM, OUTLIER>, NT, smem, g.T);
-    compress_nd_kernel<T, NDIM, OUTLIER><<<grid, NT, smem, st>>>(
+    const unsigned grid = persistent_grid(compress_nd_kernel<T, NDIM, OUTLIER>, NT_COMP, smem, g.T);
+    compress_nd_kernel<T, NDIM, OUTLIER><<<grid, NT_COMP, smem, st>>>(
         static_cast<const T *>(d_in), g, eb, eb_mode == CSZP2_EB_REL ? 1 : 0,
         static_cast<uint8_t *>(d_out), ticket, d_out_bytes, hs);
     return launch_status();

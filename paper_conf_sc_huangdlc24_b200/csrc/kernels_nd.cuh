@@ -153,238 +153,265 @@ constexpr uint32_t ND_STAGE = BPT * 4 * LND + 64;  // max tile payload + slack (
 constexpr uint32_t ND_TILE_MAX = BPT * 4 * LND;      // largest tile payload (Plain, fl = 31)
 constexpr uint32_t ND_RING = 96 * 1024;              // compression staging ring (>= ND_TILE_MAX)
 
-// Persistent compression CTAs (2 per SM), one thread per 64-value block, tiles claimed
-// in order from an atomic ticket. The decoupled lookback of a tile is DEFERRED by one
-// tile: iteration k encodes and stages tile t_k and publishes its aggregate, then
-// finishes the lookback of t_{k-1} (its window loads were issued at the end of iteration
-// k-1, so their latency hid behind t_k's gather and encode) and writes t_{k-1}'s payload
-// from the staging ring. A claimed tile therefore never waits on any lookback before
-// publishing its aggregate (no deadlock: every predecessor publishes unconditionally),
-// and no CTA idles on the inclusive-prefix round trip. When the ring cannot hold both
-// payloads, t_{k-1} is resolved and written first.
+// Warp-specialised persistent compression CTAs (NT_COMP = 288 threads: 8 producer warps,
+// one thread per 64-value block, + 1 resolver warp; 2 CTAs per SM), the same structure
+// as the 1D compress_kernel: producer thread 0 claims tiles in order from an atomic
+// ticket (after staging the previous one, so a claimed tile never waits on a lookback
+// before it publishes) and hands the ticket over through an mbarrier; the producers
+// gather their blocks straight from global memory (16-byte rows for interior blocks),
+// encode, scan (one named barrier), publish the aggregate, stage the payload in the
+// shared byte ring (byte-exact, no clearing) and queue the tile; the resolver warp runs
+// each queued tile's decoupled lookback and copies its payload out, in order. No CTA-wide
+// barrier waits on a lookback (round 1 ran it in warp 0 between two __syncthreads).
+constexpr uint32_t ND_RING_V = 128 * 1024;  // virtual lap of the ring (a power of 2 >= ND_RING)
+
 template <typename T, int NDIM, bool OUTLIER>
-__global__ void __launch_bounds__(NT, 2) compress_nd_kernel(const T *__restrict__ in, const GeomND g,
-                                                            const double eb_abs_arg,
-                                                            const int eb_from_header,
-                                                            uint8_t *__restrict__ out,
-                                                            unsigned *__restrict__ ticket,
-                                                            uint64_t *__restrict__ d_out_bytes,
-                                                            const HdrStatic hs) {
+__global__ void __launch_bounds__(NT_COMP, 2) compress_nd_kernel(const T *__restrict__ in, const GeomND g,
+                                                                 const double eb_abs_arg,
+                                                                 const int eb_from_header,
+                                                                 uint8_t *__restrict__ out,
+                                                                 unsigned *__restrict__ ticket,
+                                                                 uint64_t *__restrict__ d_out_bytes,
+                                                                 const HdrStatic hs) {
     extern __shared__ uint8_t stage_raw[];
     uint8_t *ring = smem_align<16>(stage_raw);
+    __shared__ uint64_t s_full;                    // thread 0 -> producers: the claimed ticket
+    __shared__ uint64_t s_staged[NQ], s_done[NQ];  // queue slots: producers -> resolver -> producers
+    __shared__ uint64_t s_qt[NQ];
+    __shared__ uint32_t s_qagg[NQ], s_qpos[NQ];
+    __shared__ uint8_t s_qbad[NQ];
     __shared__ uint32_t s_warp[2][NT / 32];  // tile_scan_1bar, by tile parity
-    __shared__ uint32_t s_tk[2];             // the claimed ticket of each iteration, by parity
-    __shared__ uint64_t s_excl;
-    __shared__ bool s_rng;
+    __shared__ uint32_t s_tailb[2];          // s_tail as thread 0 acquired it before the scan, by parity
+    __shared__ uint32_t s_tail;              // ring bytes released by the resolver
+    __shared__ uint32_t s_tkin;
+    __shared__ volatile uint32_t s_end;  // queue index of the end marker
     const int tid = threadIdx.x;
+    const int warp = tid >> 5, lane = tid & 31;
     const uint64_t T_eff = g.T ? g.T : 1;
     uint64_t *index = reinterpret_cast<uint64_t *>(out + 64);
     const double eb_abs =
         eb_from_header ? *reinterpret_cast<const volatile double *>(out + 32) : eb_abs_arg;
-    const auto K = make_consts(eb_abs, static_cast<T *>(nullptr));
 
-    // the deferred tile (uniform in the CTA): its number, aggregate, range flag and
-    // ring position; warp 0 also holds its lookback window
-    bool have_prev = false;
-    uint64_t prev_t = 0;
-    uint32_t prev_agg = 0, prev_pos = 0;
-    bool prev_bad = false;
-    LookbackWindow w;
-
-    // resolve the deferred tile (warp 0: lookback; tile 0 / no index: 0), write its
-    // payload from the ring, and for the last tile the pads, header and d_out_bytes.
-    // claim_slot >= 0: thread 0 then claims the next tile into s_tk[claim_slot] — after
-    // the lookback, so a claimed tile never waits on one before it publishes.
-    auto flush_prev = [&](int claim_slot) {
-        if (tid < 32) {
-            bool rng = prev_bad;
-            uint64_t e = 0;
-            if (g.T && prev_t > 0) e = lookback_finish(index, prev_t, prev_agg, prev_bad, w, &rng);
-            if (tid == 0) {
-                s_excl = e;
-                s_rng = rng;
-                if (claim_slot >= 0) s_tk[claim_slot] = atomicAdd(ticket, 1u);
-            }
+    if (tid == 0) {
+        s_end = 0xFFFFFFFFu;
+        s_tail = 0;
+        mbar_init(&s_full, 1);
+        for (int i = 0; i < NQ; i++) {
+            mbar_init(&s_staged[i], NT / 32);
+            mbar_init(&s_done[i], 1);
         }
-        __syncthreads();  // s_excl (and the ticket) visible; the deferred tile's ring bytes complete
-        const uint64_t dst0 = g.D + s_excl;
-        write_payload(ring + (prev_pos % ND_RING), out, dst0, prev_agg, tid, NT);
-        if (prev_t == T_eff - 1) {  // last tile: pads, header, d_out_bytes
-            const uint64_t dst1 = dst0 + prev_agg;
-            if (tid >= 32 && tid < 48) {
-                const uint64_t o = dst1 + (tid - 32);
-                if (o < roundup16(dst1)) out[o] = 0;
-            }
-            if (tid >= 64 && tid < 80) {
-                const uint64_t o = g.O + g.nb + (tid - 64);
-                if (o < g.D) out[o] = 0;
-            }
-            if (tid == 0) {
-                const uint32_t status = s_rng ? ST_RANGE : 0u;
-                const uint64_t pb = status ? 0 : s_excl + prev_agg;
-                const uint64_t total = roundup16(g.D + pb);
-                uint64_t *h = reinterpret_cast<uint64_t *>(out);
-                h[0] = MAGIC | (static_cast<uint64_t>(hs.word1) << 32);
-                h[1] = hs.eb_mode | (status << 8) | (static_cast<uint64_t>(BPT) << 16) |
-                       (static_cast<uint64_t>(NDIM - 1) << 32);
-                h[2] = g.n;
-                h[3] = static_cast<uint64_t>(__double_as_longlong(hs.eb_user));
-                h[4] = static_cast<uint64_t>(__double_as_longlong(eb_abs));
-                h[5] = pb;
-                h[6] = total;
-                h[7] = g.nx | (g.ny << 32);
-                if (d_out_bytes) *d_out_bytes = total;
-            }
-        }
-        __syncthreads();  // the ring bytes and s_excl are free again
-        have_prev = false;
-    };
-
-    if (tid == 0) s_tk[0] = atomicAdd(ticket, 1u);  // in-order tiles: forward progress
+        fence_mbar_init();
+        s_tkin = atomicAdd(ticket, 1u);  // in-order tiles: forward progress
+        mbar_arrive(&s_full);
+    }
     __syncthreads();
-    for (uint32_t it = 0;; ++it) {
-        const uint64_t t = s_tk[it & 1];
-        if (t >= T_eff) break;
 
-        const uint64_t b = t * BPT + tid;
-        const bool active = b < g.nb;
-        // ---- gather + ❶ quantize; values outside the field stay 0 and get residual 0
-        int q[LND];
-        uint64_t outside = 0;  // bit i: value i lies outside the field
-        bool bad = false;
-        const BlockOrigin bo = block_origin<NDIM>(g, active ? b : 0);
-        if (active && interior_vec<T, NDIM>(g, bo)) {
-            // interior block: each row of BX values by 16-byte loads
-            using S = BlockShape<NDIM>;
-            using VT = typename Vec16<T>::type;
-            constexpr int V = Vec16<T>::V;
+    if (warp < RESOLVE_WARP) {
+        // ============================== producers
+        const auto K = make_consts(eb_abs, static_cast<T *>(nullptr));
+        uint32_t head = 0;  // ring allocation cursor, identical in every producer thread
+        for (uint32_t it = 0;; ++it) {
+            const int qs = it % NQ;
+            if (tid == 0) s_tailb[it & 1] = ld_acquire_cta(&s_tail);  // handed over by the scan barrier
+            mbar_wait(&s_full, it & 1);
+            const uint64_t t = s_tkin;
+            if (t >= T_eff) {  // end marker for the resolver (one arrival per warp)
+                if (lane == 0) {
+                    if (it >= NQ) mbar_wait(&s_done[qs], (it / NQ - 1) & 1);
+                    if (tid == 0) s_end = it;
+                    mbar_arrive(&s_staged[qs]);
+                }
+                break;
+            }
+            const uint64_t b = t * BPT + tid;
+            const bool active = b < g.nb;
+            // ---- gather + ❶ quantize; values outside the field stay 0 and get residual 0
+            int q[LND];
+            uint64_t outside = 0;  // bit i: value i lies outside the field
+            bool bad = false;
+            const BlockOrigin bo = block_origin<NDIM>(g, active ? b : 0);
+            if (active && interior_vec<T, NDIM>(g, bo)) {
+                // interior block: each row of BX values by 16-byte loads
+                using S = BlockShape<NDIM>;
+                using VT = typename Vec16<T>::type;
+                constexpr int V = Vec16<T>::V;
 #pragma unroll
-            for (int r = 0; r < S::BY * S::BZ; r++) {
-                const int iy = r % S::BY, iz = r / S::BY;
-                const VT *row = reinterpret_cast<const VT *>(
-                    in + ((bo.z0 + iz) * g.ny + bo.y0 + iy) * g.nx + bo.x0);
+                for (int r = 0; r < S::BY * S::BZ; r++) {
+                    const int iy = r % S::BY, iz = r / S::BY;
+                    const VT *row = reinterpret_cast<const VT *>(
+                        in + ((bo.z0 + iz) * g.ny + bo.y0 + iy) * g.nx + bo.x0);
 #pragma unroll
-                for (int v = 0; v < S::BX / V; v++) {
-                    T tmp[V];
-                                        *reinterpret_cast<VT *>(tmp) = __ldg(row + v);
+                    for (int v = 0; v < S::BX / V; v++) {
+                        T tmp[V];
+                        *reinterpret_cast<VT *>(tmp) = __ldg(row + v);
 #pragma unroll
-                    for (int k = 0; k < V; k++) q[r * S::BX + v * V + k] = quantize_nd<NDIM>(tmp[k], K.inv, bad);
+                        for (int k = 0; k < V; k++) q[r * S::BX + v * V + k] = quantize_nd<NDIM>(tmp[k], K.inv, bad);
+                    }
+                }
+            } else {
+#pragma unroll
+                for (int i = 0; i < LND; i++) {
+                    const uint64_t idx = active ? nd_index<NDIM>(g, bo, i) : ~uint64_t(0);
+                    q[i] = 0;
+                    if (idx != ~uint64_t(0))
+                        q[i] = quantize_nd<NDIM>(in[idx], K.inv, bad);
+                    else
+                        outside |= 1ull << i;
                 }
             }
-        } else {
+            // ---- nD Lorenzo residuals, highest index first so every prediction still sees q
+            uint32_t a[LND];
+            uint64_t sign = 0;
+            uint32_t or_rest = 0;
 #pragma unroll
-            for (int i = 0; i < LND; i++) {
-                const uint64_t idx = active ? nd_index<NDIM>(g, bo, i) : ~uint64_t(0);
-                q[i] = 0;
-                if (idx != ~uint64_t(0))
-                    q[i] = quantize_nd<NDIM>(in[idx], K.inv, bad);
+            for (int i = LND - 1; i >= 0; i--) {
+                int d = q[i] - lorenzo_pred<NDIM>(q, i);
+                if ((outside >> i) & 1ull) d = 0;
+                a[i] = static_cast<uint32_t>(d < 0 ? -d : d);
+                sign |= static_cast<uint64_t>(d < 0) << i;
+                if (i) or_rest |= a[i];
+            }
+            // ---- ❷ FLE with 8-byte fields
+            const int fl_p = 32 - __clz(or_rest | a[0]);
+            uint32_t size = fl_p ? 8u * (1u + fl_p) : 0u;
+            uint32_t obyte = static_cast<uint32_t>(fl_p);
+            int fl = fl_p, nob = 0;
+            if (OUTLIER) {
+                const int fl_o = 32 - __clz(or_rest);
+                const int ob = max(1, (32 - __clz(a[0]) + 7) >> 3);
+                const uint32_t size_o = 8u + ob + 8u * fl_o;
+                if (size_o < size) {
+                    size = size_o;
+                    obyte = 0x80u | (static_cast<uint32_t>(ob - 1) << 5) | static_cast<uint32_t>(fl_o);
+                    fl = fl_o;
+                    nob = ob;
+                }
+            }
+            if (!active) {
+                size = 0;
+                bad = false;
+            }
+            if (!K.ok) bad = true;
+
+            // ---- ❸ intra-tile scan (one barrier among the producers, with the range
+            //      flag); publish the aggregate at once
+            uint32_t agg;
+            bool any_bad;
+            const uint32_t my_excl = tile_scan_1bar(size, bad, s_warp[it & 1], &agg, &any_bad, BAR_PROD);
+            if (tid == 0 && g.T) publish_aggregate(index, t, agg, any_bad);
+            if (active) out[g.O + b] = static_cast<uint8_t>(obyte);
+
+            // ---- ring room (16-aligned region, no lap straddle); the cursor thread 0
+            //      acquired before the barrier, else spin with acquire loads
+            uint32_t pos = (head + 15u) & ~15u;
+            if ((pos % ND_RING_V) + agg > ND_RING) pos = (pos / ND_RING_V + 1) * ND_RING_V;
+            auto fits = [&](uint32_t tl) { return pos + agg <= tl + ND_RING_V || tl == head; };
+            if (!fits(s_tailb[it & 1]))
+                while (!fits(ld_acquire_cta(&s_tail))) __nanosleep(64);
+            head = pos + agg;
+
+            // ---- payload into the ring: sign (8 B), outlier (nob B), planes (8 B each:
+            //      values 0..31 then 32..63), bit planes by two in-register transposes
+            const uint32_t outl = a[0];
+            if (OUTLIER && nob) a[0] = 0;
+            uint32_t(&lo)[32] = *reinterpret_cast<uint32_t(*)[32]>(&a[0]);   // values 0..31
+            uint32_t(&hi)[32] = *reinterpret_cast<uint32_t(*)[32]>(&a[32]);  // values 32..63
+            const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, static_cast<unsigned>(size ? fl : 0)));
+            if (flw > 0) {
+                if (flw <= 4) {
+                    pack_planes<2>(lo);
+                    pack_planes<2>(hi);
+                } else if (flw <= 8) {
+                    pack_planes<3>(lo);
+                    pack_planes<3>(hi);
+                } else if (flw <= 16) {
+                    pack_planes<4>(lo);
+                    pack_planes<4>(hi);
+                } else {
+                    pack_planes<5>(lo);
+                    pack_planes<5>(hi);
+                }
+            }
+            if (size) {
+                uint8_t *stg = ring + (pos % ND_RING_V);
+                if (flw <= 4)
+                    stage_payload_nd<4>(stg, my_excl, sign, outl, nob, fl, lo, hi);
+                else if (flw <= 8)
+                    stage_payload_nd<8>(stg, my_excl, sign, outl, nob, fl, lo, hi);
+                else if (flw <= 16)
+                    stage_payload_nd<16>(stg, my_excl, sign, outl, nob, fl, lo, hi);
                 else
-                    outside |= 1ull << i;
+                    stage_payload_nd<32>(stg, my_excl, sign, outl, nob, fl, lo, hi);
+            }
+
+            // ---- queue the tile (one arrival per warp; thread 0 fills in the slot)
+            __syncwarp();
+            if (lane == 0) {
+                if (it >= NQ) mbar_wait(&s_done[qs], (it / NQ - 1) & 1);  // queue slot free
+                if (tid == 0) {
+                    s_qt[qs] = t;
+                    s_qagg[qs] = agg;
+                    s_qbad[qs] = any_bad;
+                    s_qpos[qs] = pos;
+                }
+                mbar_arrive(&s_staged[qs]);
+            }
+            // ---- claim the next tile (nothing unpublished is held now)
+            if (tid == 0) {
+                s_tkin = atomicAdd(ticket, 1u);
+                mbar_arrive(&s_full);
             }
         }
-        // ---- nD Lorenzo residuals, highest index first so every prediction still sees q
-        uint32_t a[LND];
-        uint64_t sign = 0;
-        uint32_t or_rest = 0;
-#pragma unroll
-        for (int i = LND - 1; i >= 0; i--) {
-            int d = q[i] - lorenzo_pred<NDIM>(q, i);
-            if ((outside >> i) & 1ull) d = 0;
-            a[i] = static_cast<uint32_t>(d < 0 ? -d : d);
-            sign |= static_cast<uint64_t>(d < 0) << i;
-            if (i) or_rest |= a[i];
-        }
-        // ---- ❷ FLE with 8-byte fields
-        const int fl_p = 32 - __clz(or_rest | a[0]);
-        uint32_t size = fl_p ? 8u * (1u + fl_p) : 0u;
-        uint32_t obyte = static_cast<uint32_t>(fl_p);
-        int fl = fl_p, nob = 0;
-        if (OUTLIER) {
-            const int fl_o = 32 - __clz(or_rest);
-            const int ob = max(1, (32 - __clz(a[0]) + 7) >> 3);
-            const uint32_t size_o = 8u + ob + 8u * fl_o;
-            if (size_o < size) {
-                size = size_o;
-                obyte = 0x80u | (static_cast<uint32_t>(ob - 1) << 5) | static_cast<uint32_t>(fl_o);
-                fl = fl_o;
-                nob = ob;
+    } else {
+        // ============================== resolver: ❸ then ❹, in tile order
+        for (uint32_t it = 0;; ++it) {
+            const int q = it % NQ;
+            mbar_wait_backoff(&s_staged[q], (it / NQ) & 1, 100);
+            if (it >= s_end) break;
+            const uint64_t t = s_qt[q];
+            const uint32_t agg = s_qagg[q];
+            const uint32_t pos = s_qpos[q];
+            const bool bad = s_qbad[q];
+            bool rng = bad;
+            uint64_t excl = 0;
+            if (g.T && t > 0) excl = lookback(index, t, agg, bad, &rng);
+            const uint64_t dst0 = g.D + excl;
+            write_payload(ring + (pos % ND_RING_V), out, dst0, agg, lane, 32);
+            if (t == T_eff - 1) {  // last tile: pads, header, d_out_bytes
+                const uint64_t dst1 = dst0 + agg;
+                __syncwarp();
+                if (lane < 16) {  // zero pad after the payload
+                    const uint64_t o = dst1 + lane;
+                    if (o < roundup16(dst1)) out[o] = 0;
+                } else {  // zero pad after the offset bytes
+                    const uint64_t o = g.O + g.nb + (lane - 16);
+                    if (o < g.D) out[o] = 0;
+                }
+                if (lane == 0) {
+                    const uint32_t status = rng ? ST_RANGE : 0u;
+                    const uint64_t pb = status ? 0 : excl + agg;
+                    const uint64_t total = roundup16(g.D + pb);
+                    uint64_t *h = reinterpret_cast<uint64_t *>(out);
+                    h[0] = MAGIC | (static_cast<uint64_t>(hs.word1) << 32);
+                    h[1] = hs.eb_mode | (status << 8) | (static_cast<uint64_t>(BPT) << 16) |
+                           (static_cast<uint64_t>(NDIM - 1) << 32);
+                    h[2] = g.n;
+                    h[3] = static_cast<uint64_t>(__double_as_longlong(hs.eb_user));
+                    h[4] = static_cast<uint64_t>(__double_as_longlong(eb_abs));
+                    h[5] = pb;
+                    h[6] = total;
+                    h[7] = g.nx | (g.ny << 32);
+                    if (d_out_bytes) *d_out_bytes = total;
+                }
+            }
+            __syncwarp();  // every lane's reads of these ring bytes are ordered before the release
+            if (lane == 0) {
+                __threadfence_block();  // release pattern: fence, then the relaxed cursor store
+                st_relaxed_cta(&s_tail, pos + agg);  // in order, so the ring frees in order
+                mbar_arrive(&s_done[q]);
             }
         }
-        if (!active) {
-            size = 0;
-            bad = false;
-        }
-        if (!K.ok) bad = true;
-
-        // ---- ❸ intra-tile scan (one barrier, with the range flag); publish the
-        //      aggregate at once (never behind a lookback)
-        uint32_t agg;
-        bool any_bad;
-        const uint32_t my_excl = tile_scan_1bar(size, bad, s_warp[it & 1], &agg, &any_bad, 0);
-        if (tid == 0 && g.T) publish_aggregate(index, t, agg, any_bad);
-        if (active) out[g.O + b] = static_cast<uint8_t>(obyte);
-
-        // ---- ring space behind the deferred tile's payload, else resolve that one first
-        uint32_t pos = have_prev ? ((prev_pos + prev_agg + 15u) & ~15u) : 0u;
-        if ((pos % ND_RING) + agg > ND_RING) pos = (pos / ND_RING + 1) * ND_RING;
-        if (have_prev && pos + agg > prev_pos + ND_RING) {
-            flush_prev(-1);
-            pos = 0;
-        }
-
-        // ---- payload into the ring: sign (8 B), outlier (nob B), planes (8 B each:
-        //      values 0..31 then 32..63), bit planes by two in-register transposes
-        const uint32_t outl = a[0];
-        if (OUTLIER && nob) a[0] = 0;
-        uint32_t(&lo)[32] = *reinterpret_cast<uint32_t(*)[32]>(&a[0]);   // values 0..31
-        uint32_t(&hi)[32] = *reinterpret_cast<uint32_t(*)[32]>(&a[32]);  // values 32..63
-        const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, static_cast<unsigned>(size ? fl : 0)));
-        if (flw > 0) {
-            if (flw <= 4) {
-                pack_planes<2>(lo);
-                pack_planes<2>(hi);
-            } else if (flw <= 8) {
-                pack_planes<3>(lo);
-                pack_planes<3>(hi);
-            } else if (flw <= 16) {
-                pack_planes<4>(lo);
-                pack_planes<4>(hi);
-            } else {
-                pack_planes<5>(lo);
-                pack_planes<5>(hi);
-            }
-        }
-        if (size) {
-            uint8_t *stg = ring + (pos % ND_RING);
-            if (flw <= 4)
-                stage_payload_nd<4>(stg, my_excl, sign, outl, nob, fl, lo, hi);
-            else if (flw <= 8)
-                stage_payload_nd<8>(stg, my_excl, sign, outl, nob, fl, lo, hi);
-            else if (flw <= 16)
-                stage_payload_nd<16>(stg, my_excl, sign, outl, nob, fl, lo, hi);
-            else
-                stage_payload_nd<32>(stg, my_excl, sign, outl, nob, fl, lo, hi);
-        }
-
-        // ---- the deferred tile: its window has been in flight since last iteration
-        //      (its first barrier also completes this tile's staging and hands out the
-        //      next ticket)
-        if (have_prev) {
-            flush_prev((it + 1) & 1);
-        } else {
-            if (tid == 0) s_tk[(it + 1) & 1] = atomicAdd(ticket, 1u);
-            __syncthreads();
-        }
-
-        // ---- this tile becomes the deferred one; issue its lookback window now
-        have_prev = true;
-        prev_t = t;
-        prev_agg = agg;
-        prev_pos = pos;
-        prev_bad = any_bad;
-        if (tid < 32 && g.T && t > 0) lookback_issue(index, static_cast<int64_t>(t) - 1, w);
     }
-    if (have_prev) flush_prev(-1);
 }
 
 template <typename T, int NDIM>
