@@ -120,3 +120,23 @@ def test_compress_slab_global_rel_world1(nccl_group):
     assert rc == oracle.OK and int(nb.item()) == s.size
     np.testing.assert_array_equal(out[: s.size].cpu().numpy(), s)
     assert offs.cpu().tolist() == [0, s.size]
+
+
+@pytest.mark.parametrize("scope", ["rank", "global"])
+def test_compress_slab_on_a_side_stream(nccl_group, scope):
+    """compress_slab(stream=s) orders the compressor, the size all-gather (NCCL) and the
+    container-index kernel on `s`: with a side stream whose queue is kept
+    busy ahead of the call, the offsets still read the stream's final size."""
+    n = 40 * 8192 + 32 * 5 + 3
+    x = make_field("cfg2", "cuda:0", 0, n)
+    side = torch.cuda.Stream()
+    busy = torch.empty(1 << 26, device="cuda:0")
+    with torch.cuda.stream(side):
+        for _ in range(8):
+            busy.mul_(1.0001)  # queue work ahead of the compressor on the side stream
+    out, nb, offs = compress_slab(x, 1e-3, "rel", "outlier", stream=side, rel_scope=scope)
+    torch.cuda.synchronize()
+    s, rc = oracle.compress(x.cpu().numpy(), 1e-3, oracle.REL, oracle.OUTLIER)
+    assert rc == oracle.OK and int(nb.item()) == s.size
+    np.testing.assert_array_equal(out[: s.size].cpu().numpy(), s)
+    assert offs.cpu().tolist() == [0, s.size]

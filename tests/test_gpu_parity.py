@@ -509,3 +509,21 @@ def test_binding_validates_buffers():
     for c in bad_calls:
         with pytest.raises(ValueError):
             c()
+
+
+@pytest.mark.parametrize("eb_mode", ["abs", "rel"])
+def test_encode_prepared_flag(eb_mode):
+    """FLAG_PREPARED (include/cszp2.h): after a prepare, encode may skip re-zeroing the
+    tile index — the stream is the oracle's; cszp2_compress uses exactly this pair."""
+    rng = np.random.default_rng(78)
+    xh = np.cumsum(rng.standard_normal(8192 * 20 + 45)).astype(np.float32)
+    x = torch.from_numpy(xh).to(DEV)
+    out = torch.full((cz.compress_bound(x.numel()),), 0xAA, dtype=torch.uint8, device=DEV)
+    nb = torch.zeros(1, dtype=torch.int64, device=DEV)
+    for enc in ("outlier", "plain"):
+        cz.compress_prepare(x, 1e-3, eb_mode, out)
+        cz.compress_encode(x, 1e-3, eb_mode, enc, out, nb, prepared=True)
+        torch.cuda.synchronize()
+        ref, rc = oracle.compress(xh, 1e-3, EBM[eb_mode], ENC[enc])
+        assert rc == oracle.OK and int(nb.item()) == ref.size
+        np.testing.assert_array_equal(out[:ref.size].cpu().numpy(), ref)
