@@ -155,3 +155,16 @@ def test_nd_persistent_multi_tile_per_cta(kind):
         rng = np.random.default_rng(12)
         xh = (rng.standard_normal(shape) * 100.0).astype(np.float32)
         check_nd(xh, 1e-5, "abs", "plain")
+
+
+@pytest.mark.parametrize("shape", [(9, 10, 128), (5, 17, 384), (3, 33, 256), (4, 4, 128), (64, 64, 512)])
+@pytest.mark.parametrize("enc", ["plain", "outlier"])
+def test_nd3_wide_rows_parity(shape, enc):
+    """3D f32 fields with long rows (x a multiple of 128, so every warp's 32 blocks are
+    one run of a block row), y/z extents that are not multiples of 4, partial last tiles,
+    many tiles per CTA, and an incompressible field (ring-full path)."""
+    xh = smooth_field(shape, sum(shape) + 5, np.float32, noise=1e-2)
+    check_nd(xh, 1e-4, "rel", enc)
+    rng = np.random.default_rng(sum(shape))
+    xn = (rng.standard_normal(shape) * 100.0).astype(np.float32)  # incompressible: direct path
+    check_nd(xn, 1e-5, "abs", enc)
