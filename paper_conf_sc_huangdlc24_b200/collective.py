@@ -36,10 +36,18 @@ class CudaCodec:
     eb_mode: str = "rel"
     enc_mode: str = "outlier"
 
-    def compress(self, x: torch.Tensor, stream=None):
-        from . import compress
+    def compress(self, x: torch.Tensor, workspace: dict | None = None, stream=None):
+        """One fused compression kernel; reuses workspace["cmp"] / ["nbytes"] when given."""
+        from . import compress, compress_bound
 
-        return compress(x, self.eb, self.eb_mode, self.enc_mode, stream=stream)
+        ws = {} if workspace is None else workspace
+        bound = compress_bound(x.numel(), x.dtype)
+        buf = ws.get("cmp")
+        if buf is None or buf.numel() < bound or buf.device != x.device:
+            buf = ws["cmp"] = torch.empty(bound, dtype=torch.uint8, device=x.device)
+            ws["nbytes"] = torch.zeros(1, dtype=torch.int64, device=x.device)
+        return compress(x, self.eb, self.eb_mode, self.enc_mode, out=buf[:bound], out_bytes=ws["nbytes"],
+                        stream=stream)
 
     def decompress(self, cmp: torch.Tensor, n: int, out: torch.Tensor, status: torch.Tensor, stream=None):
         """Decode into `out`; `status` (zeroed device int32) receives FORMAT/RANGE bits."""
@@ -58,10 +66,13 @@ def _all_gather_bytes(recv: torch.Tensor, send: torch.Tensor, group=None):
 
 
 def compressed_all_gather(x: torch.Tensor, eb: float, eb_mode: str = "rel", enc_mode: str = "outlier",
-                          group=None, codec=None, out: torch.Tensor | None = None, stats: dict | None = None):
+                          group=None, codec=None, out: torch.Tensor | None = None, stats: dict | None = None,
+                          workspace: dict | None = None):
     """All-gather equal-sized shards through the compressor. Returns a tensor of
     world·n values (rank order), like all_gather_into_tensor of the lossy shards.
-    `stats` (optional dict) receives the per-rank stream sizes and wire bytes."""
+    `stats` (optional dict) receives the per-rank stream sizes and wire bytes.
+    `workspace` (optional dict, kept by the caller across calls) holds the compressed
+    buffer, the receive buffer and the status words, so repeated calls allocate nothing."""
     codec = codec or CudaCodec(eb, eb_mode, enc_mode)
     x = x.contiguous().view(-1)
     world = dist.get_world_size(group)
@@ -70,14 +81,22 @@ def compressed_all_gather(x: torch.Tensor, eb: float, eb_mode: str = "rel", enc_
         raise ValueError("shard size must be a multiple of 16 bytes (output slices stay 16-byte aligned)")
     if out is None:
         out = torch.empty(world * n, dtype=x.dtype, device=x.device)
-    buf, nbytes = codec.compress(x)                 # 1. one fused compression kernel
+    ws = {} if workspace is None else workspace
+    buf, nbytes = codec.compress(x, ws)             # 1. one fused compression kernel
     sizes = gather_sizes(nbytes.view(1), group)     # 2. 8 B per rank over NCCL
     slot = (int(sizes.max().item()) + 15) // 16 * 16  # the one host read
     if slot > buf.numel():
         raise RuntimeError("compressed stream larger than its buffer")
-    recv = torch.empty(world * slot, dtype=torch.uint8, device=x.device)
+    recv = ws.get("recv")
+    if recv is None or recv.numel() < world * slot or recv.device != x.device:
+        recv = ws["recv"] = torch.empty(world * slot, dtype=torch.uint8, device=x.device)
+    recv = recv[: world * slot]
     _all_gather_bytes(recv, buf[:slot], group)      # 3. the compressed payloads
-    status = torch.zeros(world, dtype=torch.int32, device=x.device)
+    status = ws.get("status")
+    if status is None or status.numel() != world or status.device != x.device:
+        status = ws["status"] = torch.zeros(world, dtype=torch.int32, device=x.device)
+    else:
+        status.zero_()
     for r in range(world):                          # 4. P decompression kernels
         codec.decompress(recv[r * slot:(r + 1) * slot], n, out[r * n:(r + 1) * n], status[r:r + 1])
     bad = [(r, int(v)) for r, v in enumerate(status.tolist()) if v]  # host sync after the decodes

@@ -52,6 +52,25 @@ from paper_conf_sc_huangdlc24_b200.multi import compress_slab, slab  # noqa: E40
 from tests import streamparse as sp  # noqa: E402
 
 
+def test_compressed_all_gather_reuses_its_workspace(nccl_group):
+    """With a caller-kept workspace, repeated calls reuse the compressed, receive and
+    status buffers (same storage) and still return the oracle's round trip."""
+    n = 3 * 8192 + 32 * 3 + 12
+    ws = {}
+    ptrs = None
+    for seed in range(3):
+        x = make_field("cfg2", "cuda:0", seed * n, n)
+        y = compressed_all_gather(x, 1e-4, "rel", "outlier", workspace=ws)
+        torch.cuda.synchronize()
+        s, rc = oracle.compress(x.cpu().numpy(), 1e-4, oracle.REL, oracle.OUTLIER)
+        yr, rc2 = oracle.decompress(s, n)
+        np.testing.assert_array_equal(y.cpu().numpy().view(np.uint32), yr.view(np.uint32))
+        p = (ws["cmp"].data_ptr(), ws["recv"].data_ptr(), ws["status"].data_ptr())
+        if ptrs is not None:
+            assert p[0] == ptrs[0] and p[2] == ptrs[2]  # same compressed buffer and status words
+        ptrs = p
+
+
 @pytest.mark.parametrize("dtype", [np.float32, np.float64])
 def test_value_range_exact(dtype):
     rng = np.random.default_rng(7)

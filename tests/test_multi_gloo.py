@@ -100,7 +100,7 @@ class _OracleCodec:
     def __init__(self, eb, eb_mode, enc):
         self.eb, self.eb_mode, self.enc = eb, eb_mode, enc
 
-    def compress(self, x):
+    def compress(self, x, workspace=None):
         import oracle
 
         s, rc = oracle.compress(x.numpy(), self.eb, self.eb_mode, self.enc)
