@@ -75,3 +75,16 @@ def test_cpu_tensors_are_rejected():
     for i, c in enumerate(calls):
         with pytest.raises(ValueError):
             c()
+
+
+def test_nd_extent_limit_matches_1d():
+    """One size limit for every entry point: nx*ny*nz <= 2^35 values, as the
+    1D n <= 2^35; beyond it the nD bound is 0 (invalid) for compression and the same
+    geometry is rejected by decompression (checked on the GPU by the ABI test)."""
+    import paper_conf_sc_huangdlc24_b200 as cz
+
+    assert cz.compress_bound_nd((2 ** 11, 2 ** 12, 2 ** 12)) > 0          # 2^35 values
+    assert cz.compress_bound_nd((2 ** 11, 2 ** 12, 2 ** 12 + 4)) == 0      # just past 2^35
+    assert cz.compress_bound_nd((2 ** 17, 2 ** 18)) > 0                    # 2D, 2^35
+    assert cz.compress_bound_nd((2 ** 17 + 1, 2 ** 18)) == 0
+    assert cz.compress_bound(2 ** 35) > 0

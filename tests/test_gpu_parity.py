@@ -448,6 +448,8 @@ def test_c_abi_rejects_invalid_arguments():
     assert L.cszp2_compress_prepare_range(p(x), 10, 0, 1e-3, None, p(out), s) == E
     assert L.cszp2_compress_prepare_range(p(x), 10, 0, 1e-3, p(out, 8), p(out), s) == E
     assert L.cszp2_compress_prepare_range(p(x), 10, 0, 0.0, p(nb), p(out), s) == E
+    assert L.cszp2_decompress_nd(p(out), p(x), 2 ** 12, 2 ** 12, 2 ** 12, 3, 0, None, s) == E  # > 2^35 values
+    assert L.cszp2_compress_nd(p(x), 2 ** 12, 2 ** 12, 2 ** 12, 3, 0, 1e-3, 0, 0, p(out), p(nb), s) == E
     torch.cuda.synchronize()
     assert int(nb.item()) == 0 and int(out.sum().item()) == 0  # nothing was written
 
