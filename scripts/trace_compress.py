@@ -31,6 +31,11 @@ for arg in sys.argv[1:]:
     claim, data, pub, res, staged, polls, rstart = [a[:, i] for i in range(7)]
     moves = np.zeros_like(polls)
     print(f"== {cfg}: T={T} span={(res.max())/1e3:.1f}us rate={T/(res.max()/1e3):.1f} tiles/us")
+    copied_ = a[:, 9]
+    print(f"ramp/tail: first data {data[data>0].min()/1e3:.2f}us, first pubA {pub.min()/1e3:.2f}us, "
+          f"1st-wave (first 444 tiles) resolved by {np.max(res[:min(T,444)])/1e3:.2f}us, "
+          f"10%/50%/90%/100% of tiles resolved at " + "/".join(f"{np.percentile(res, p)/1e3:.2f}" for p in (10, 50, 90, 100))
+          + f"us, last copy {copied_.max()/1e3:.2f}us, last claim {claim.max()/1e3:.2f}us")
     def q(v): return " ".join(f"{np.percentile(v,p):7.2f}" for p in (5,25,50,75,95,99))
     print("pct                5      25      50      75      95      99  (us)")
     print("claim->data   ", q((data-claim)/1e3))
