@@ -249,14 +249,22 @@ int geometry_nd(uint64_t nx, uint64_t ny, uint64_t nz, int ndim, GeomND *g) {
     g->T = (g->nb + BPT - 1) / BPT;
     g->O = roundup16(64 + 8 * g->T);
     g->D = roundup16(g->O + g->nb);
+    g->dbx = make_fastdiv(static_cast<uint32_t>(g->nbx ? g->nbx : 1));
+    g->dby = make_fastdiv(static_cast<uint32_t>(g->nby ? g->nby : 1));
     return CSZP2_OK;
 }
 uint64_t stream_bound_nd(const GeomND &g) { return roundup16(g.D + static_cast<uint64_t>(4 * LND) * g.nb); }
 
 template <typename T, int NDIM, bool OUTLIER>
-int launch_compress_nd(const void *d_in, const GeomND &g, double eb, int eb_mode, int enc_mode,
+int launch_compress_nd(const void *d_in, const GeomND &g0, double eb, int eb_mode, int enc_mode,
                        void *d_out, uint64_t *d_out_bytes, cudaStream_t st) {
     constexpr int smem = ND_RING + 64;
+    GeomND g = g0;  // + the gather strides of this value type
+    const uint64_t by = NDIM == 2 ? 8 : 4;  // block rows r = iy + by * iz
+    for (int r = 0; r < 16; r++) g.roff[r] = ((r / by) * g.ny + (r % by)) * g.nx * sizeof(T);
+    g.ystep = g.roff[1];
+    g.zstep = NDIM == 3 ? g.roff[4] - g.roff[3] : 0;
+    g.vec = (g.nx % (16 / sizeof(T))) == 0 ? 1u : 0u;
     if (int rc = set_smem(compress_nd_kernel<T, NDIM, OUTLIER>, smem)) return rc;
     unsigned *ticket = reinterpret_cast<unsigned *>(static_cast<uint8_t *>(d_out) + stream_bound_nd(g));
     HdrStatic hs;
@@ -552,3 +560,10 @@ int cszp2_container_index(const uint64_t *d_sizes, int nparts, uint64_t *d_offse
 }
 
 }  // extern "C"
+
+#ifdef CSZP2_WD
+// debug build only: point the kernels' watchdog records at host-mapped memory
+extern "C" int cszp2_debug_watch(void *p) {
+    return cudaMemcpyToSymbol(cszp2::g_wd, &p, sizeof(p)) == cudaSuccess ? CSZP2_OK : CSZP2_ERR_CUDA;
+}
+#endif

@@ -37,6 +37,25 @@ __device__ __forceinline__ uint64_t gtimer() {
 #define TRACE(tile, slot, val) do { } while (0)
 #endif
 
+#ifdef CSZP2_WD
+// debug build only (hang hunting): spinning sites report their state into host-mapped
+// memory, 8 records of 8 words per CTA, read by the host while the kernel runs
+__device__ uint64_t *g_wd = nullptr;
+#define WD_REC(site, a, b, c, d)                                                          \
+    do {                                                                                  \
+        if (g_wd) {                                                                       \
+            volatile uint64_t *r_ = g_wd + (static_cast<uint64_t>(blockIdx.x) * 8 + (site)) * 8; \
+            r_[1] = (a);                                                                  \
+            r_[2] = (b);                                                                  \
+            r_[3] = (c);                                                                  \
+            r_[4] = (d);                                                                  \
+            r_[0] = (site) | (static_cast<uint64_t>(threadIdx.x) << 8) | (1ull << 40);    \
+        }                                                                                 \
+    } while (0)
+#else
+#define WD_REC(site, a, b, c, d) do { } while (0)
+#endif
+
 constexpr int L = 32;      // values per block
 constexpr int BPT = 256;   // blocks per tile (FORMAT.md §1)
 constexpr int NT = 256;    // threads per CTA: one block per thread
@@ -493,6 +512,13 @@ __device__ __forceinline__ uint64_t lookback_finish(uint64_t *index, uint64_t t,
         const uint32_t P = __reduce_min_sync(0xffffffffu, pk);
         const uint32_t W = __reduce_min_sync(0xffffffffu, wk);
         if (W < P) {  // a needed predecessor is still Waiting: re-poll the Waiting slots
+#ifdef CSZP2_WD
+            {
+                static_assert(true, "");
+                const uint64_t wd_t = t;
+                if (lane == 0) WD_REC(6, wd_t, static_cast<uint64_t>(j), P, (static_cast<uint64_t>(W) << 32) | (t - 1 - j + W));
+            }
+#endif
 #ifdef CSZP2_TRACE
             if (lane == 0 && g_trace) g_trace[t * 16 + 5]++;
 #endif

@@ -13,10 +13,35 @@ namespace cszp2 {
 
 constexpr int LND = 64;  // values per multi-dimensional block
 
+// Exact u32 division by a runtime constant for dividends < 2^31 (round-up multiplier,
+// Granlund & Montgomery): q = umulhi(n, m) >> s, with m = ceil(2^(31+l) / d),
+// l = ceil(log2 d); d = 1 is the identity (m = 0).
+struct FastDiv {
+    uint32_t d, m, s;
+};
+__host__ __device__ inline FastDiv make_fastdiv(uint32_t d) {
+    FastDiv f{d, 0u, 0u};
+    if (d > 1) {
+        uint32_t l = 0;
+        while ((1ull << l) < d) l++;
+        const uint32_t p = 31 + l;
+        f.m = static_cast<uint32_t>(((1ull << p) + d - 1) / d);
+        f.s = p - 32;
+    }
+    return f;
+}
+__device__ __forceinline__ uint32_t fast_div(uint32_t n, const FastDiv &f) {
+    return f.d == 1 ? n : (__umulhi(n, f.m) >> f.s);
+}
+
 struct GeomND {
     uint64_t nx, ny, nz;    // field extents, x fastest
     uint64_t nbx, nby, nbz; // block grid
     uint64_t n, nb, T, O, D;
+    FastDiv dbx, dby;       // division by nbx, nby (used while nb < 2^31)
+    uint64_t roff[16];      // compression gathers: byte offset of block row r (r = iy + BY iz)
+    uint64_t ystep, zstep;  // the same as steps: row r-1 -> r within / across a z-plane
+    uint32_t vec;           // rows are whole 16-byte vectors (nx % (16/w) == 0)
 };
 
 template <int NDIM>
@@ -105,6 +130,134 @@ __device__ __forceinline__ bool interior_vec(const GeomND &g, const BlockOrigin 
     return (g.nx % Vec16<T>::V) == 0 && o.x0 + S::BX <= g.nx && o.y0 + S::BY <= g.ny &&
            o.z0 + S::BZ <= g.nz;
 }
+
+// ❶ for one value, as a BIASED pattern (f32: q + 0x4B400000 mod 2^32; f64: q).
+// UNCHECKED (f32 only): the bits of fl(x·inv + 1.5·2^23), exact whenever the block passes
+// the certificate in compress_nd_kernel; CHECKED: FORMAT.md §7's range check.
+template <int NDIM, bool CHECKED>
+__device__ __forceinline__ uint32_t qpattern(float x, float inv, bool &bad) {
+    const float t = __fmul_rn(x, inv);
+    if (!CHECKED) return static_cast<uint32_t>(__float_as_int(__fadd_rn(t, 12582912.0f)));
+    bad |= !(fabsf(t) <= (NDIM == 2 ? 268435440.0f : 134217720.0f));
+    return static_cast<uint32_t>(__float2int_rn(t)) + 0x4B400000u;
+}
+template <int NDIM, bool CHECKED>
+__device__ __forceinline__ uint32_t qpattern(double x, double inv, bool &bad) {
+    const double t = __dmul_rn(x, inv);
+    bad |= !(fabs(t) <= (NDIM == 2 ? 268435455.0 : 134217727.0));
+    return static_cast<uint32_t>(__double_as_longlong(__dadd_rn(t, 6755399441055744.0)));  // rint(t), |t| < 2^31
+}
+
+// Gather + ❶ of the 64 values of block origin bo, row by row (3D: 16 rows of 4, 2D: 8
+// rows of 8 values), each row from base + roff[r] (host-computed byte offsets). Interior
+// blocks of fields whose rows are whole 16-byte vectors load unpredicated vectors; edge
+// blocks the same vectors predicated on lying inside the field; other fields (nx not a
+// multiple of the vector width) value by value. Values outside the field (and every
+// value of an inactive block) get the pattern of q = 0 and bit i of *outside.
+template <typename T, int NDIM, bool CHECKED>
+__device__ __forceinline__ void gather_block(const T *__restrict__ in, const GeomND &g, uint32_t x0, uint32_t y0,
+                                             uint32_t z0, bool active, T inv, uint32_t (&v)[LND],
+                                             uint64_t &outside, bool &bad) {
+    using S = BlockShape<NDIM>;
+    using VT = typename Vec16<T>::type;
+    constexpr int V = Vec16<T>::V;
+    constexpr int NROW = LND / S::BX;
+    const char *base =
+        reinterpret_cast<const char *>(in) + ((static_cast<uint64_t>(z0) * g.ny + y0) * g.nx + x0) * sizeof(T);
+    uint64_t outb = 0;
+    if (g.vec) {
+        const bool interior = active && x0 + S::BX <= g.nx && y0 + S::BY <= g.ny && z0 + S::BZ <= g.nz;
+        if (interior) {
+            // rows by a chain of pointer steps (so that the 16 row addresses are never
+            // all live at once: 64 values + 32 address registers would spill)
+            const char *rp = base;
+#pragma unroll
+            for (int r = 0; r < NROW; r++) {
+                // f64: at most 32 loaded registers in flight (all 128 would spill)
+                if (sizeof(T) == 8 && r && (r * S::BX) % 16 == 0) asm volatile("" ::: "memory");
+                if (r) rp += (r % S::BY) ? g.ystep : g.zstep;
+                const VT *row = reinterpret_cast<const VT *>(rp);
+#pragma unroll
+                for (int u = 0; u < S::BX / V; u++) {
+                    T tmp[V];
+                    *reinterpret_cast<VT *>(tmp) = __ldg(row + u);
+#pragma unroll
+                    for (int k = 0; k < V; k++) v[r * S::BX + u * V + k] = qpattern<NDIM, CHECKED>(tmp[k], inv, bad);
+                }
+            }
+        } else {
+#pragma unroll
+            for (int r = 0; r < NROW; r++) {
+                if (sizeof(T) == 8 && r && (r * S::BX) % 16 == 0) asm volatile("" ::: "memory");
+                const uint32_t dy = r % S::BY, dz = r / S::BY;
+                const bool row_ok = active && y0 + dy < g.ny && z0 + dz < g.nz;
+                const VT *row = reinterpret_cast<const VT *>(base + g.roff[r]);
+#pragma unroll
+                for (int u = 0; u < S::BX / V; u++) {
+                    const bool ok = row_ok && x0 + u * V < g.nx;  // nx % V == 0: whole vectors
+                    T tmp[V];
+#pragma unroll
+                    for (int k = 0; k < V; k++) tmp[k] = T(0);
+                    if (ok) *reinterpret_cast<VT *>(tmp) = __ldg(row + u);
+                    outb |= static_cast<uint64_t>(ok ? 0u : (1u << V) - 1u) << (r * S::BX + u * V);
+#pragma unroll
+                    for (int k = 0; k < V; k++) v[r * S::BX + u * V + k] = qpattern<NDIM, CHECKED>(tmp[k], inv, bad);
+                }
+            }
+        }
+    } else {
+#pragma unroll
+        for (int r = 0; r < NROW; r++) {
+            if (r && (r * S::BX) % 16 == 0) asm volatile("" ::: "memory");
+            const uint32_t dy = r % S::BY, dz = r / S::BY;
+            const bool row_ok = active && y0 + dy < g.ny && z0 + dz < g.nz;
+            const T *row = reinterpret_cast<const T *>(base + g.roff[r]);
+#pragma unroll
+            for (int ix = 0; ix < S::BX; ix++) {
+                const bool ok = row_ok && x0 + ix < g.nx;
+                const T val = ok ? row[ix] : T(0);
+                outb |= static_cast<uint64_t>(!ok) << (r * S::BX + ix);
+                v[r * S::BX + ix] = qpattern<NDIM, CHECKED>(val, inv, bad);
+            }
+        }
+    }
+    outside = outb;
+}
+
+// nD Lorenzo residuals of the biased patterns, in place: the separable product of first
+// differences along x, y (and z) with in-block zero boundaries, which expands to q - pred
+// with FORMAT.md §7's 3- / 7-neighbour prediction ((1-S_x)(1-S_y)(1-S_z) q). The biases
+// cancel in every difference except at the block's corner (value 0, no neighbour).
+// Cost per 64 values: 112 (2D) / 144 (3D) integer subtractions.
+template <typename T, int NDIM>
+__device__ __forceinline__ void lorenzo_block(uint32_t (&v)[LND]) {
+    using S = BlockShape<NDIM>;
+    constexpr int NROW = LND / S::BX;
+#pragma unroll
+    for (int r = 0; r < NROW; r++)
+#pragma unroll
+        for (int ix = S::BX - 1; ix >= 1; ix--) v[r * S::BX + ix] -= v[r * S::BX + ix - 1];
+#pragma unroll
+    for (int z = 0; z < S::BZ; z++)
+#pragma unroll
+        for (int iy = S::BY - 1; iy >= 1; iy--)
+#pragma unroll
+            for (int ix = 0; ix < S::BX; ix++)
+                v[(z * S::BY + iy) * S::BX + ix] -= v[(z * S::BY + iy - 1) * S::BX + ix];
+    if (NDIM == 3) {
+#pragma unroll
+        for (int z = S::BZ - 1; z >= 1; z--)
+#pragma unroll
+            for (int m = 0; m < S::BX * S::BY; m++) v[z * S::BX * S::BY + m] -= v[(z - 1) * S::BX * S::BY + m];
+    }
+    v[0] -= static_cast<uint32_t>(QBias<T>::value);
+}
+// f32 certificate for the unchecked patterns: a block whose residuals all have |d| < 2^15
+// has |q| <= 64 (2^15 - 1) < 2^22 everywhere (q is the in-block box sum of at most 64
+// residuals, modulo 2^32 as computed), so every pattern lies strictly inside the binade
+// where the RN addition is rint(t) exactly and |t| < 2^22 passes the range check (the 1D
+// kernel's argument, quantize_block_unchecked); NaN and ±Inf fall outside it.
+constexpr int ND_FAST_FL_MAX = 15;
 
 // One block's nD payload (FORMAT.md §7: sign 8 B, nob outlier bytes, then planes
 // k = 0..fl-1 as (lo word, hi word)) to smem at byte `st` (any alignment). With the
@@ -225,52 +378,65 @@ __global__ void __launch_bounds__(NT_COMP, 2) compress_nd_kernel(const T *__rest
             }
             const uint64_t b = t * BPT + tid;
             const bool active = b < g.nb;
-            // ---- gather + ❶ quantize; values outside the field stay 0 and get residual 0
-            int q[LND];
-            uint64_t outside = 0;  // bit i: value i lies outside the field
-            bool bad = false;
-            const BlockOrigin bo = block_origin<NDIM>(g, active ? b : 0);
-            if (active && interior_vec<T, NDIM>(g, bo)) {
-                // interior block: each row of BX values by 16-byte loads
+            uint32_t x0, y0, z0;  // block origin (every extent is < 2^32)
+            {
                 using S = BlockShape<NDIM>;
-                using VT = typename Vec16<T>::type;
-                constexpr int V = Vec16<T>::V;
+                const uint64_t bb = active ? b : 0;
+                uint32_t cbx, cby, cbz;
+                if (g.nb < (1ull << 31)) {
+                    const uint32_t r32 = fast_div(static_cast<uint32_t>(bb), g.dbx);
+                    const uint32_t z32 = fast_div(r32, g.dby);
+                    cbx = static_cast<uint32_t>(bb) - r32 * static_cast<uint32_t>(g.nbx);
+                    cby = r32 - z32 * static_cast<uint32_t>(g.nby);
+                    cbz = z32;
+                } else {
+                    const uint64_t r = bb / g.nbx, z = r / g.nby;
+                    cbx = static_cast<uint32_t>(bb - r * g.nbx);
+                    cby = static_cast<uint32_t>(r - z * g.nby);
+                    cbz = static_cast<uint32_t>(z);
+                }
+                x0 = cbx * S::BX;
+                y0 = cby * S::BY;
+                z0 = cbz * S::BZ;
+            }
+            // ---- gather + ❶ (f32: unchecked patterns, redone checked if the block fails the
+            //      certificate) + nD Lorenzo residuals
+            uint32_t v[LND];
+            uint64_t outside;
+            bool bad = false;
+            uint32_t(&a)[LND] = v;  // residual magnitudes, in place
+            uint32_t sign_lo = 0, sign_hi = 0, or_rest = 0;
+            auto residuals = [&]() {
+                lorenzo_block<T, NDIM>(v);
+                if (outside) {  // values outside the field have residual 0 (FORMAT.md §7)
 #pragma unroll
-                for (int r = 0; r < S::BY * S::BZ; r++) {
-                    const int iy = r % S::BY, iz = r / S::BY;
-                    const VT *row = reinterpret_cast<const VT *>(
-                        in + ((bo.z0 + iz) * g.ny + bo.y0 + iy) * g.nx + bo.x0);
+                    for (int i = 0; i < LND; i++)
+                        if ((outside >> i) & 1ull) v[i] = 0;
+                }
+                or_rest = 0;
 #pragma unroll
-                    for (int v = 0; v < S::BX / V; v++) {
-                        T tmp[V];
-                        *reinterpret_cast<VT *>(tmp) = __ldg(row + v);
-#pragma unroll
-                        for (int k = 0; k < V; k++) q[r * S::BX + v * V + k] = quantize_nd<NDIM>(tmp[k], K.inv, bad);
-                    }
+                for (int i = LND - 1; i >= 0; i--) {
+                    const int d = static_cast<int>(v[i]);
+                    a[i] = static_cast<uint32_t>(d < 0 ? -d : d);
+                    if (i >= 32)
+                        sign_hi = __funnelshift_l(static_cast<uint32_t>(d), sign_hi, 1);  // bit i-32 = d_i < 0
+                    else
+                        sign_lo = __funnelshift_l(static_cast<uint32_t>(d), sign_lo, 1);
+                    if (i) or_rest |= a[i];
+                }
+            };
+            if (sizeof(T) == 4) {
+                gather_block<T, NDIM, false>(in, g, x0, y0, z0, active, K.inv, v, outside, bad);
+                residuals();
+                if (32 - __clz(or_rest | a[0]) > ND_FAST_FL_MAX) {
+                    gather_block<T, NDIM, true>(in, g, x0, y0, z0, active, K.inv, v, outside, bad);
+                    residuals();
                 }
             } else {
-#pragma unroll
-                for (int i = 0; i < LND; i++) {
-                    const uint64_t idx = active ? nd_index<NDIM>(g, bo, i) : ~uint64_t(0);
-                    q[i] = 0;
-                    if (idx != ~uint64_t(0))
-                        q[i] = quantize_nd<NDIM>(in[idx], K.inv, bad);
-                    else
-                        outside |= 1ull << i;
-                }
+                gather_block<T, NDIM, true>(in, g, x0, y0, z0, active, K.inv, v, outside, bad);
+                residuals();
             }
-            // ---- nD Lorenzo residuals, highest index first so every prediction still sees q
-            uint32_t a[LND];
-            uint64_t sign = 0;
-            uint32_t or_rest = 0;
-#pragma unroll
-            for (int i = LND - 1; i >= 0; i--) {
-                int d = q[i] - lorenzo_pred<NDIM>(q, i);
-                if ((outside >> i) & 1ull) d = 0;
-                a[i] = static_cast<uint32_t>(d < 0 ? -d : d);
-                sign |= static_cast<uint64_t>(d < 0) << i;
-                if (i) or_rest |= a[i];
-            }
+            const uint64_t sign = static_cast<uint64_t>(sign_lo) | (static_cast<uint64_t>(sign_hi) << 32);
             // ---- ❷ FLE with 8-byte fields
             const int fl_p = 32 - __clz(or_rest | a[0]);
             uint32_t size = fl_p ? 8u * (1u + fl_p) : 0u;
@@ -317,31 +483,33 @@ __global__ void __launch_bounds__(NT_COMP, 2) compress_nd_kernel(const T *__rest
             uint32_t(&lo)[32] = *reinterpret_cast<uint32_t(*)[32]>(&a[0]);   // values 0..31
             uint32_t(&hi)[32] = *reinterpret_cast<uint32_t(*)[32]>(&a[32]);  // values 32..63
             const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, static_cast<unsigned>(size ? fl : 0)));
-            if (flw > 0) {
-                if (flw <= 4) {
-                    pack_planes<2>(lo);
-                    pack_planes<2>(hi);
-                } else if (flw <= 8) {
-                    pack_planes<3>(lo);
-                    pack_planes<3>(hi);
-                } else if (flw <= 16) {
-                    pack_planes<4>(lo);
-                    pack_planes<4>(hi);
-                } else {
-                    pack_planes<5>(lo);
-                    pack_planes<5>(hi);
-                }
-            }
-            if (size) {
-                uint8_t *stg = ring + (pos % ND_RING_V);
-                if (flw <= 4)
-                    stage_payload_nd<4>(stg, my_excl, sign, outl, nob, fl, lo, hi);
-                else if (flw <= 8)
-                    stage_payload_nd<8>(stg, my_excl, sign, outl, nob, fl, lo, hi);
-                else if (flw <= 16)
-                    stage_payload_nd<16>(stg, my_excl, sign, outl, nob, fl, lo, hi);
-                else
-                    stage_payload_nd<32>(stg, my_excl, sign, outl, nob, fl, lo, hi);
+            uint8_t *stg = ring + (pos % ND_RING_V);
+            if (flw == 0) {
+                if (size) stage_payload_nd<0>(stg, my_excl, sign, outl, nob, 0, lo, hi);
+            } else if (flw <= 1) {
+                pack_planes<0>(lo);
+                pack_planes<0>(hi);
+                if (size) stage_payload_nd<1>(stg, my_excl, sign, outl, nob, fl, lo, hi);
+            } else if (flw <= 2) {
+                pack_planes<1>(lo);
+                pack_planes<1>(hi);
+                if (size) stage_payload_nd<2>(stg, my_excl, sign, outl, nob, fl, lo, hi);
+            } else if (flw <= 4) {
+                pack_planes<2>(lo);
+                pack_planes<2>(hi);
+                if (size) stage_payload_nd<4>(stg, my_excl, sign, outl, nob, fl, lo, hi);
+            } else if (flw <= 8) {
+                pack_planes<3>(lo);
+                pack_planes<3>(hi);
+                if (size) stage_payload_nd<8>(stg, my_excl, sign, outl, nob, fl, lo, hi);
+            } else if (flw <= 16) {
+                pack_planes<4>(lo);
+                pack_planes<4>(hi);
+                if (size) stage_payload_nd<16>(stg, my_excl, sign, outl, nob, fl, lo, hi);
+            } else {
+                pack_planes<5>(lo);
+                pack_planes<5>(hi);
+                if (size) stage_payload_nd<32>(stg, my_excl, sign, outl, nob, fl, lo, hi);
             }
 
             // ---- queue the tile (one arrival per warp; thread 0 fills in the slot)
