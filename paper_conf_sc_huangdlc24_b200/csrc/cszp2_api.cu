@@ -255,16 +255,22 @@ int geometry_nd(uint64_t nx, uint64_t ny, uint64_t nz, int ndim, GeomND *g) {
 }
 uint64_t stream_bound_nd(const GeomND &g) { return roundup16(g.D + static_cast<uint64_t>(4 * LND) * g.nb); }
 
+// byte offsets of the block rows (r = iy + by * iz) for the nD gathers / scatters
+template <typename T, int NDIM>
+void nd_rows(GeomND &g) {
+    const uint64_t by = NDIM == 2 ? 8 : 4;
+    for (int r = 0; r < 16; r++) g.roff[r] = ((r / by) * g.ny + (r % by)) * g.nx * sizeof(T);
+    g.ystep = g.roff[1];
+    g.zstep = NDIM == 3 ? g.roff[4] - g.roff[3] : 0;
+    g.vec = (g.nx % (16 / sizeof(T))) == 0 ? 1u : 0u;
+}
+
 template <typename T, int NDIM, bool OUTLIER>
 int launch_compress_nd(const void *d_in, const GeomND &g0, double eb, int eb_mode, int enc_mode,
                        void *d_out, uint64_t *d_out_bytes, cudaStream_t st) {
     constexpr int smem = ND_RING + 64;
     GeomND g = g0;  // + the gather strides of this value type
-    const uint64_t by = NDIM == 2 ? 8 : 4;  // block rows r = iy + by * iz
-    for (int r = 0; r < 16; r++) g.roff[r] = ((r / by) * g.ny + (r % by)) * g.nx * sizeof(T);
-    g.ystep = g.roff[1];
-    g.zstep = NDIM == 3 ? g.roff[4] - g.roff[3] : 0;
-    g.vec = (g.nx % (16 / sizeof(T))) == 0 ? 1u : 0u;
+    nd_rows<T, NDIM>(g);
     if (int rc = set_smem(compress_nd_kernel<T, NDIM, OUTLIER>, smem)) return rc;
     unsigned *ticket = reinterpret_cast<unsigned *>(static_cast<uint8_t *>(d_out) + stream_bound_nd(g));
     HdrStatic hs;
@@ -281,14 +287,25 @@ int launch_compress_nd(const void *d_in, const GeomND &g0, double eb, int eb_mod
 }
 
 template <typename T, int NDIM>
-int launch_decompress_nd(const void *d_cmp, void *d_out, const GeomND &g, int *d_status,
+int launch_decompress_nd(const void *d_cmp, void *d_out, const GeomND &g0, int *d_status,
                          cudaStream_t st) {
-    constexpr int smem = ND_STAGE + 64;
-    if (int rc = set_smem(decompress_nd_kernel<T, NDIM>, smem)) return rc;
-    const unsigned grid = static_cast<unsigned>(g.T ? g.T : 1);
-    decompress_nd_kernel<T, NDIM><<<grid, NT, smem, st>>>(static_cast<const uint8_t *>(d_cmp),
-                                                          static_cast<T *>(d_out), g, d_status);
-    return launch_status();
+    if constexpr (sizeof(T) == 8) {  // f64: one CTA per tile (kernels_nd.cuh, decompress_nd_tile_kernel)
+        constexpr int smem = ND_STAGE + 64;
+        if (int rc = set_smem(decompress_nd_tile_kernel<T, NDIM>, smem)) return rc;
+        const unsigned grid = static_cast<unsigned>(g0.T ? g0.T : 1);
+        decompress_nd_tile_kernel<T, NDIM><<<grid, NT, smem, st>>>(static_cast<const uint8_t *>(d_cmp),
+                                                                   static_cast<T *>(d_out), g0, d_status);
+        return launch_status();
+    } else {
+        constexpr int smem = ND_DRING + 64;
+        if (int rc = set_smem(decompress_nd_kernel<T, NDIM>, smem)) return rc;
+        GeomND g = g0;
+        nd_rows<T, NDIM>(g);
+        const unsigned grid = persistent_grid(decompress_nd_kernel<T, NDIM>, NT, smem, g.T);
+        decompress_nd_kernel<T, NDIM><<<grid, NT, smem, st>>>(static_cast<const uint8_t *>(d_cmp),
+                                                              static_cast<T *>(d_out), g, d_status);
+        return launch_status();
+    }
 }
 
 template <typename T>

@@ -582,8 +582,336 @@ __global__ void __launch_bounds__(NT_COMP, 2) compress_nd_kernel(const T *__rest
     }
 }
 
+// Inverse of lorenzo_block: in-block prefix sums along x, y (and z) of the residuals
+// (mod 2^32), i.e. q = box sum of d — the separable form of q_i = d_i + pred_i in index
+// order (FORMAT.md §7); 112 (2D) / 144 (3D) integer additions per block. The last
+// direction's sums run row by row and each finished row is handed to emit(r) at once, so
+// that the stores spread over the arithmetic instead of leaving in one burst.
+template <int NDIM, typename Emit>
+__device__ __forceinline__ void inv_lorenzo_block(uint32_t (&v)[LND], Emit &&emit) {
+    using S = BlockShape<NDIM>;
+    constexpr int NROW = LND / S::BX;
+#pragma unroll
+    for (int r = 0; r < NROW; r++)
+#pragma unroll
+        for (int ix = 1; ix < S::BX; ix++) v[r * S::BX + ix] += v[r * S::BX + ix - 1];
+    if (NDIM == 2) {
+#pragma unroll
+        for (int iy = 0; iy < S::BY; iy++) {
+            if (iy)
+#pragma unroll
+                for (int ix = 0; ix < S::BX; ix++) v[iy * S::BX + ix] += v[(iy - 1) * S::BX + ix];
+            emit(iy);
+        }
+    } else {
+#pragma unroll
+        for (int z = 0; z < S::BZ; z++)
+#pragma unroll
+            for (int iy = 1; iy < S::BY; iy++)
+#pragma unroll
+                for (int ix = 0; ix < S::BX; ix++)
+                    v[(z * S::BY + iy) * S::BX + ix] += v[(z * S::BY + iy - 1) * S::BX + ix];
+#pragma unroll
+        for (int z = 0; z < S::BZ; z++) {
+            if (z)
+#pragma unroll
+                for (int m = 0; m < S::BX * S::BY; m++) v[z * S::BX * S::BY + m] += v[(z - 1) * S::BX * S::BY + m];
+#pragma unroll
+            for (int iy = 0; iy < S::BY; iy++) emit(z * S::BY + iy);
+        }
+    }
+}
+
+constexpr uint32_t ND_DRING = 96 * 1024;  // decompression payload ring per CTA (2 x 64 KiB + 16 do not fit:
+                                         // the next payload goes behind the current one or waits)
+
+// Persistent decompression CTAs (256 threads, one per 64-value block; 2 per SM): CTA c
+// decodes tiles c, c + G, ...; each tile's payload range comes from the persisted tile
+// index in O(1) (R-14) and is bulk-loaded (1D TMA) into a 96 KiB ring while the previous
+// tile is decoded (the 1D decompress_kernel's scheme: behind the current payload, else
+// at the ring's start, else deferred until the ring is empty); index words and offset
+// bytes are fetched two tiles ahead. Per block: scan of the 256 sizes, sign / outlier /
+// two 32x32 plane transposes (values 0..31, 32..63), prefix sums (inverse Lorenzo),
+// I2FP + FMUL, 16-byte streaming row stores (edge blocks value by value, bounds-checked).
 template <typename T, int NDIM>
-__global__ void __launch_bounds__(NT, 3) decompress_nd_kernel(const uint8_t *__restrict__ cmp,
+__global__ void __launch_bounds__(NT, 2) decompress_nd_kernel(const uint8_t *__restrict__ cmp, T *__restrict__ out,
+                                                           const GeomND g, int *__restrict__ d_status) {
+    extern __shared__ uint8_t stage_raw[];
+    uint8_t *ring = smem_align<16>(stage_raw);
+    __shared__ uint64_t s_bar[2];
+    __shared__ uint32_t s_warp[NT / 32];
+    __shared__ uint64_t s_excl[2];
+    __shared__ uint32_t s_bytes[2];
+    __shared__ uint32_t s_rpos[2];
+    __shared__ double s_eb;
+    __shared__ int s_err;
+    using S = BlockShape<NDIM>;
+    const int tid = threadIdx.x;
+    const uint64_t G = gridDim.x;
+    const uint64_t *index = reinterpret_cast<const uint64_t *>(cmp) + 8;
+    constexpr uint32_t BAD_BYTES = 0xFFFFFFFFu;
+    uint64_t raw_p = FLAG_P, raw_i = 0, pb_hdr = 0;
+    bool pending = false, deferred = false;
+    uint32_t r_pos = 0, r_len = 0;
+    auto launch = [&](uint64_t dp, uint64_t di, int bi, bool ring_empty) -> bool {
+        const uint64_t e = dp & VAL_MASK, i = di & VAL_MASK;
+        uint32_t bytes = BAD_BYTES;
+        if ((dp >> 61) == 4 && (di >> 61) == 4 && i >= e && i <= pb_hdr && i - e <= static_cast<uint64_t>(BPT) * 4 * LND)
+            bytes = static_cast<uint32_t>(i - e);
+        s_excl[bi] = e;
+        s_bytes[bi] = bytes;
+        if (bytes != BAD_BYTES && bytes) {
+            const uint64_t src0 = (g.D + e) & ~uint64_t(15);
+            const uint32_t len = static_cast<uint32_t>(roundup16(g.D + e + bytes) - src0);
+            uint32_t pos;
+            if (ring_empty)
+                pos = 0;
+            else if (r_pos + r_len + len <= ND_DRING - 16)
+                pos = r_pos + r_len;
+            else if (len + 16 <= r_pos)
+                pos = 0;
+            else
+                return false;
+            s_rpos[bi] = pos;
+            r_pos = pos;
+            r_len = len;
+            mbar_expect_tx(&s_bar[bi], len);
+            bulk_load(ring + pos, cmp + src0, len, &s_bar[bi]);
+        } else {
+            s_rpos[bi] = 0;
+            r_len = 0;
+            mbar_expect_tx(&s_bar[bi], 0);
+        }
+        return true;
+    };
+
+    uint64_t t = blockIdx.x;
+    if (tid == 0) {
+        const uint64_t *h = reinterpret_cast<const uint64_t *>(cmp);
+        const uint64_t h0 = h[0], h1 = h[1];
+        int err = 0;
+        const uint32_t want1 = 1u | (static_cast<uint32_t>(Traits<T>::DTYPE) << 8) | (6u << 24);
+        if ((h0 & 0xFFFFFFFFu) != MAGIC || ((h0 >> 32) & 0xFF00FFFFu) != want1 ||
+            ((h1 >> 16) & 0xFFFFu) != BPT || ((h1 >> 32) & 0xFFu) != static_cast<uint64_t>(NDIM - 1) ||
+            h[2] != g.n || h[7] != (g.nx | (g.ny << 32)))
+            err = ST_FORMAT;
+        else if (((h1 >> 8) & 0xFF) != 0)
+            err = ((h1 >> 8) & 0xFF) == ST_RANGE ? ST_RANGE : ST_FORMAT;
+        pb_hdr = h[5];
+        if (!err && h[6] != roundup16(g.D + pb_hdr)) err = ST_FORMAT;
+        s_err = err;
+        s_eb = __longlong_as_double(static_cast<long long>(h[4]));
+        mbar_init(&s_bar[0], 1);
+        mbar_init(&s_bar[1], 1);
+        fence_mbar_init();
+        if (!err && t < g.T) {
+            launch(t ? index[t - 1] : FLAG_P, index[t], 0, true);
+            pending = true;
+            const uint64_t t2 = t + G;
+            if (t2 < g.T) {
+                raw_p = index[t2 - 1];
+                raw_i = index[t2];
+            }
+        }
+    }
+    __syncthreads();
+    if (s_err) {
+        if (tid == 0 && d_status) atomicOr(d_status, s_err);
+        return;
+    }
+    const auto K = make_consts(s_eb, static_cast<T *>(nullptr));
+    uint32_t ob_cur = 0, ob_next = 0;
+    {
+        const uint64_t b = t * BPT + tid;
+        if (t < g.T && b < g.nb) ob_cur = cmp[g.O + b];
+        const uint64_t bn = (t + G) * BPT + tid;
+        if (t + G < g.T && bn < g.nb) ob_next = cmp[g.O + bn];
+    }
+    int err = 0;
+    for (uint32_t it = 0; t < g.T; ++it, t += G) {
+        const int cur = it & 1;
+        const uint64_t tn = t + G;
+        uint64_t nraw_p = 0, nraw_i = 0;
+        if (tid == 0) {
+            pending = false;
+            deferred = false;
+            if (tn < g.T) {  // the next tile's payload streams in during this one
+                nraw_p = raw_p;
+                nraw_i = raw_i;
+                deferred = !launch(raw_p, raw_i, cur ^ 1, false);
+                pending = !deferred;
+                const uint64_t t2 = tn + G;
+                if (t2 < g.T) {
+                    raw_p = index[t2 - 1];
+                    raw_i = index[t2];
+                }
+            }
+        }
+        uint32_t ob_pref = 0;  // offset byte of tile t + 2G
+        {
+            const uint64_t t2 = tn + G;
+            const uint64_t b2 = t2 * BPT + tid;
+            if (t2 < g.T && b2 < g.nb) ob_pref = cmp[g.O + b2];
+        }
+        const uint64_t b = t * BPT + tid;
+        const bool active = b < g.nb;
+        const uint32_t obyte = ob_cur;
+        const uint32_t fl = obyte & 31u;
+        const bool is_o = (obyte & 0x80u) != 0;
+        const uint32_t nob = is_o ? ((obyte >> 5) & 3u) + 1u : 0u;
+        const bool bad = (!is_o && (obyte & 0x60u));
+        const uint32_t size = is_o ? 8u + nob + 8u * fl : (fl ? 8u * (1u + fl) : 0u);
+        // one-barrier scan: s_warp is next rewritten after the CTA barrier below
+        uint32_t agg;
+        bool any_bad;
+        const uint32_t my_excl = tile_scan_1bar(size, bad, s_warp, &agg, &any_bad, 0);
+        if (any_bad || agg != s_bytes[cur]) {
+            err = ST_FORMAT;
+            if (tid == 0) {
+                mbar_wait(&s_bar[cur], (it >> 1) & 1);
+                if (pending) mbar_wait(&s_bar[cur ^ 1], ((it + 1) >> 1) & 1);
+            }
+            break;
+        }
+        mbar_wait(&s_bar[cur], (it >> 1) & 1);
+
+        // ---- ❷⁻¹: sign (8 B), outlier, planes (8 B each) -> residual magnitudes
+        uint32_t v[LND];
+        uint32_t(&lo)[32] = *reinterpret_cast<uint32_t(*)[32]>(&v[0]);
+        uint32_t(&hi)[32] = *reinterpret_cast<uint32_t(*)[32]>(&v[32]);
+        uint32_t sign_lo = 0, sign_hi = 0, outl = 0;
+        const int flw = static_cast<int>(__reduce_max_sync(0xffffffffu, size ? fl : 0u));
+        {
+            const uint8_t *pbuf = ring + s_rpos[cur];
+            uint32_t p = static_cast<uint32_t>((g.D + s_excl[cur]) & 15u) + my_excl;
+            if (size) {
+                sign_lo = ld_u32_unaligned(pbuf, p);
+                sign_hi = ld_u32_unaligned(pbuf, p + 4);
+                p += 8;
+                if (is_o) {
+                    outl = ld_u32_unaligned(pbuf, p);
+                    if (nob < 4) outl &= (1u << (8 * nob)) - 1u;
+                    p += nob;
+                }
+            }
+            // plane k = (lo word, hi word) at p + 8k: one funnel of two aligned words each
+            const uint32_t *w = reinterpret_cast<const uint32_t *>(pbuf + (p & ~3u));
+            const uint32_t sh = 8u * (p & 3u);
+            auto planes = [&](auto RC) {
+                constexpr int R = decltype(RC)::value;
+                uint32_t prev = size ? w[0] : 0u;
+#pragma unroll
+                for (int k = 0; k < R; k++) {
+                    uint32_t l = 0, hh = 0;
+                    if (size && k < (int)fl) {
+                        const uint32_t w1 = w[2 * k + 1], w2 = w[2 * k + 2];
+                        l = __funnelshift_r(prev, w1, sh);
+                        hh = __funnelshift_r(w1, w2, sh);
+                        prev = w2;
+                    }
+                    lo[k] = l;
+                    hi[k] = hh;
+                }
+#pragma unroll
+                for (int k = R; k < 32; k++) lo[k] = hi[k] = 0;
+            };
+            if (flw == 0) {
+#pragma unroll
+                for (int k = 0; k < 32; k++) lo[k] = hi[k] = 0;
+            } else if (flw <= 1) {
+                planes(std::integral_constant<int, 1>());
+                unpack_planes<0>(lo);
+                unpack_planes<0>(hi);
+            } else if (flw <= 2) {
+                planes(std::integral_constant<int, 2>());
+                unpack_planes<1>(lo);
+                unpack_planes<1>(hi);
+            } else if (flw <= 4) {
+                planes(std::integral_constant<int, 4>());
+                unpack_planes<2>(lo);
+                unpack_planes<2>(hi);
+            } else if (flw <= 8) {
+                planes(std::integral_constant<int, 8>());
+                unpack_planes<3>(lo);
+                unpack_planes<3>(hi);
+            } else if (flw <= 16) {
+                planes(std::integral_constant<int, 16>());
+                unpack_planes<4>(lo);
+                unpack_planes<4>(hi);
+            } else {
+                planes(std::integral_constant<int, 32>());
+                unpack_planes<5>(lo);
+                unpack_planes<5>(hi);
+            }
+        }
+        __syncthreads();  // every thread has read this tile's payload from the ring
+        if (tid == 0 && deferred) {  // the ring is empty now: fetch the next payload
+            launch(nraw_p, nraw_i, cur ^ 1, true);
+            pending = true;
+        }
+        if (is_o) lo[0] = outl;
+#pragma unroll
+        for (int i = 0; i < 32; i++) {
+            if ((sign_lo >> i) & 1u) lo[i] = 0u - lo[i];
+            if ((sign_hi >> i) & 1u) hi[i] = 0u - hi[i];
+        }
+        // ---- inverse Lorenzo (residuals -> q), ❶⁻¹ and the stores, row by row
+        uint32_t x0 = 0, y0 = 0, z0 = 0;
+        if (active) {
+            uint32_t cbx, cby, cbz;
+            if (g.nb < (1ull << 31)) {
+                const uint32_t r32 = fast_div(static_cast<uint32_t>(b), g.dbx);
+                const uint32_t z32 = fast_div(r32, g.dby);
+                cbx = static_cast<uint32_t>(b) - r32 * static_cast<uint32_t>(g.nbx);
+                cby = r32 - z32 * static_cast<uint32_t>(g.nby);
+                cbz = z32;
+            } else {
+                const uint64_t r = b / g.nbx, z = r / g.nby;
+                cbx = static_cast<uint32_t>(b - r * g.nbx);
+                cby = static_cast<uint32_t>(r - z * g.nby);
+                cbz = static_cast<uint32_t>(z);
+            }
+            x0 = cbx * S::BX;
+            y0 = cby * S::BY;
+            z0 = cbz * S::BZ;
+        }
+        char *base = reinterpret_cast<char *>(out) + ((static_cast<uint64_t>(z0) * g.ny + y0) * g.nx + x0) * sizeof(T);
+        const bool interior = active && g.vec && x0 + S::BX <= g.nx && y0 + S::BY <= g.ny && z0 + S::BZ <= g.nz;
+        char *rp = base;
+        inv_lorenzo_block<NDIM>(v, [&](int r) {
+            if (interior) {
+                using VT = typename Vec16<T>::type;
+                constexpr int V = Vec16<T>::V;
+                if (r) rp += (r % S::BY) ? g.ystep : g.zstep;
+#pragma unroll
+                for (int u = 0; u < S::BX / V; u++) {
+                    T tmp[V];
+#pragma unroll
+                    for (int k = 0; k < V; k++) tmp[k] = dequantize(static_cast<int>(v[r * S::BX + u * V + k]), K.s);
+                    __stcs(reinterpret_cast<VT *>(rp) + u, *reinterpret_cast<VT *>(tmp));
+                }
+            } else if (active) {
+                const uint32_t dy = r % S::BY, dz = r / S::BY;
+                const bool row_ok = y0 + dy < g.ny && z0 + dz < g.nz;
+                T *row = reinterpret_cast<T *>(base + g.roff[r]);
+#pragma unroll
+                for (int ix = 0; ix < S::BX; ix++)
+                    if (row_ok && x0 + ix < g.nx) row[ix] = dequantize(static_cast<int>(v[r * S::BX + ix]), K.s);
+            }
+        });
+        ob_cur = ob_next;
+        ob_next = ob_pref;
+    }
+    if (tid == 0 && err && d_status) atomicOr(d_status, err);
+}
+
+// One CTA per tile (3 per SM; grid = tiles), the round-1/2 decompressor, kept for f64:
+// there its 24 warps per SM and value-order inverse Lorenzo (each value stored as soon as
+// it is final) sustain the store stream better than the persistent kernel's 16 warps
+// with 32 16-byte stores per thread per tile (0.266 vs 0.315 ms on config 4b, 512^3 f64;
+// profiles/ab_nd_r03j.txt: long-scoreboard waits on the stores' source registers).
+template <typename T, int NDIM>
+__global__ void __launch_bounds__(NT, 3) decompress_nd_tile_kernel(const uint8_t *__restrict__ cmp,
                                                            T *__restrict__ out, const GeomND g,
                                                            int *__restrict__ d_status) {
     extern __shared__ uint8_t stage_raw[];

@@ -168,3 +168,30 @@ def test_nd3_wide_rows_parity(shape, enc):
     rng = np.random.default_rng(sum(shape))
     xn = (rng.standard_normal(shape) * 100.0).astype(np.float32)  # incompressible: direct path
     check_nd(xn, 1e-5, "abs", enc)
+
+
+@pytest.mark.parametrize("shape", [(96, 136), (12, 40, 68)])
+@pytest.mark.parametrize("enc", ["plain", "outlier"])
+@pytest.mark.parametrize("sigma_q", [2.0 ** 11, 2.0 ** 12.5, 2.0 ** 13.5])
+def test_nd_certificate_boundary(shape, enc, sigma_q):
+    """f32 nD compression quantizes with the unchecked magic-add patterns and redoes a
+    block with F2I when its residuals reach |d| >= 2^15 (kernels_nd.cuh, ND_FAST_FL_MAX):
+    noise scaled so that the blocks' fixed lengths straddle 15/16/17 must still give the
+    oracle's stream byte for byte."""
+    rng = np.random.default_rng(int(sigma_q) + len(shape))
+    eb = 1e-3
+    xh = (rng.standard_normal(shape) * sigma_q * 2 * eb).astype(np.float32)
+    check_nd(xh, eb, "abs", enc)
+
+
+@pytest.mark.parametrize("ndim", [2, 3])
+@pytest.mark.parametrize("offset_q", [2.0 ** 20, 2.0 ** 21.5, 2.0 ** 22, 2.0 ** 23.5])
+def test_nd_large_q_small_residuals(ndim, offset_q):
+    """Smooth fields riding on a large offset: |q| from 2^20 to 2^23.5 (around the 2^22
+    edge of the fast quantizer's binade) with small in-block residuals except at each
+    block's corner, Outlier and Plain: streams and values equal the oracle's."""
+    shape = (64, 72) if ndim == 2 else (16, 20, 24)
+    eb = 1e-4
+    xh = (smooth_field(shape, 3, np.float64, noise=1e-4) + offset_q * 2 * eb).astype(np.float32)
+    for enc in ("plain", "outlier"):
+        check_nd(xh, eb, "abs", enc)
