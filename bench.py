@@ -550,7 +550,8 @@ def run_config_sweep(args, cz, dev, stream, peak, clk):
     """Every other BASELINE config on one GPU (BASELINE.md "Output"):
     config x REL bound x encoding mode, both directions, device-timed with CUDA events
     on the launching stream, L2 flushed (a 256 MiB write) before every timed
-    direction, since configs 1-3a fit in the 126 MB L2."""
+    direction, since configs 1-3a fit in the 126 MB L2, and a device spin before each
+    step so that host launch latency never shows up between the events."""
     rows = []
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     for cfg in SWEEP:
@@ -567,6 +568,10 @@ def run_config_sweep(args, cz, dev, stream, peak, clk):
                 for k in range(3 + K):  # 3 untimed warm-up steps
                     e = ev[k - 3] if k >= 3 else None
                     flush.zero_()
+                    # ~0.2 ms device spin: the host enqueues the whole step before the GPU
+                    # reaches e[0], so the events time the kernels back to back, not the
+                    # host's launch latency (which exceeds a small config's kernel time)
+                    torch.cuda._sleep(400_000)
                     if e: e[0].record(stream)
                     cz.compress_prepare(x, eb, spec.eb_mode, out, stream=stream)
                     if e: e[1].record(stream)

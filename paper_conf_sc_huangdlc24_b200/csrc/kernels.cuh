@@ -723,7 +723,10 @@ __global__ void __launch_bounds__(256) minmax_kernel(const T *__restrict__ in, u
 }
 
 // The same reduction with the field streamed through shared memory by 1D bulk TMA
-// copies (MM_STAGES chunks of 16 KiB per CTA in flight; CTA c takes chunks c, c+G, ...):
+// copies (MM_STAGES chunks of 16 KiB per CTA in flight; CTA c takes chunks c, c+G, ...,
+// counted from the END of the field, so that the field's first ~100 MB — the tiles the
+// compressor claims first, right after this pass — are the most recently read and still
+// in the 126 MB L2):
 // bulk copies keep ~128 KiB per SM in flight with no load instructions, which the
 // register-staged loop above cannot (it tops out near 6.6 TB/s, this near the HBM read
 // rate). d_in is 16-byte aligned (cszp2_compress contract); the bytes past the last
@@ -758,7 +761,7 @@ __global__ void __launch_bounds__(256) minmax_kernel_tma(const T *__restrict__ i
             const uint64_t c = blockIdx.x + static_cast<uint64_t>(k) * gridDim.x;
             if (c < nchunks) {
                 mbar_expect_tx(&s_full[k], MM_CHUNK);
-                bulk_load(mm_smem + k * MM_CHUNK, src + c * MM_CHUNK, MM_CHUNK, &s_full[k]);
+                bulk_load(mm_smem + k * MM_CHUNK, src + (nchunks - 1 - c) * MM_CHUNK, MM_CHUNK, &s_full[k]);
             }
         }
     }
@@ -783,7 +786,7 @@ __global__ void __launch_bounds__(256) minmax_kernel_tma(const T *__restrict__ i
         const uint64_t cn = c + static_cast<uint64_t>(MM_STAGES) * gridDim.x;
         if (tid == 0 && cn < nchunks) {
             mbar_expect_tx(&s_full[k], MM_CHUNK);
-            bulk_load(mm_smem + k * MM_CHUNK, src + cn * MM_CHUNK, MM_CHUNK, &s_full[k]);
+            bulk_load(mm_smem + k * MM_CHUNK, src + (nchunks - 1 - cn) * MM_CHUNK, MM_CHUNK, &s_full[k]);
         }
     }
     if (blockIdx.x == 0) {  // values past the last whole chunk
