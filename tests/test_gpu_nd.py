@@ -195,3 +195,36 @@ def test_nd_large_q_small_residuals(ndim, offset_q):
     xh = (smooth_field(shape, 3, np.float64, noise=1e-4) + offset_q * 2 * eb).astype(np.float32)
     for enc in ("plain", "outlier"):
         check_nd(xh, eb, "abs", enc)
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_nd_decompress_rejects_corrupt_streams(dtype):
+    """FORMAT errors inside a multi-tile 3D stream (an offset byte with reserved bits, an
+    offset byte whose size no longer sums to the tile's index range, a cleared index
+    flag) in the first and in a later tile: status FORMAT (4), and the decompressor
+    returns (its payload prefetch in flight is drained, no hang)."""
+    shape = (64, 64, 96)  # 6144 blocks = 24 tiles, several per persistent CTA
+    xh = smooth_field(shape, 9, dtype, noise=1e-2)
+    x, out, total = gpu_nd(xh, 1e-4, "rel", "outlier")
+    nb = (64 // 4) * (64 // 4) * (96 // 4)
+    T = -(-nb // 256)
+    O = (64 + 8 * T + 15) // 16 * 16
+
+    def status(buf):
+        st = torch.zeros(1, dtype=torch.int32, device=DEV)
+        cz.decompress_nd(buf, shape, x.dtype, status=st)
+        torch.cuda.synchronize()
+        return int(st.item())
+
+    assert status(out) == 0
+    for b in (3, 256 * 17 + 5):
+        bad = out.clone()
+        bad[O + b] = 0x60  # Plain block with the reserved bits set
+        assert status(bad) == 4
+        bad = out.clone()
+        bad[O + b] = (int(out[O + b].item()) & 0xE0) | ((int(out[O + b].item()) + 1) & 31)  # size changes
+        assert status(bad) == 4
+    for t in (0, 13):
+        bad = out.clone()
+        bad[64 + 8 * t + 7] = 0  # descriptor flag cleared
+        assert status(bad) == 4
