@@ -2,10 +2,13 @@
 // §VI-D / Table VI: 2D Lorenzo on 8x8 blocks and 3D Lorenzo on 4x4x4
 // blocks (L = 64), same Plain/Outlier FLE, same decoupled-lookback concatenation
 // (FORMAT.md §7). The paper keeps them out of the main design because they cost
-// throughput (>50%). Compression: persistent CTAs claiming tiles in order from
-// an atomic ticket, one thread per 64-value block, values gathered straight from
-// global memory (16-byte rows), the lookback deferred by one tile. Decompression: one
-// CTA per tile, the payload located in O(1) by the tile index and bulk-loaded.
+// throughput (>50%). Compression: warp-specialised persistent CTAs (8 producer
+// warps, one thread per 64-value block, values gathered straight from global memory by
+// 16-byte rows and quantized with the 1D kernel's unchecked magic-add under a per-block
+// certificate; separable Lorenzo; 1 resolver warp for lookback + copy-out) claiming tiles
+// in order from an atomic ticket. Decompression: f32 — persistent CTAs with the payload
+// ring prefetch of the 1D kernel and row-by-row inverse Lorenzo + stores; f64 — one CTA
+// per tile (decompress_nd_tile_kernel). DESIGN.md §6.
 #pragma once
 #include "kernels.cuh"
 
