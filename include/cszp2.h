@@ -127,6 +127,9 @@ int cszp2_compress_prepare_range(const void *d_in, uint64_t n, int dtype, double
  *  CSZP2_FLAG_LOAD_SCALAR: each thread loads its block value by value (the
  *    non-vectorised baseline of the §VI-E memory ablation).
  *  LOAD_VEC and LOAD_SCALAR are exclusive (ARG otherwise).
+ *  CSZP2_FLAG_LB_WIDE / CSZP2_FLAG_LB_NARROW: force the lookback's first window
+ *    to 256 / 32 predecessors (by default 32 up to 2^17 tiles, 256 beyond; a speed
+ *    choice that changes no stream byte). Exclusive (ARG otherwise).
  *  CSZP2_FLAG_PREPARED (not an ablation): the caller guarantees that a
  *    cszp2_compress_prepare(_range) on this d_out precedes this call on the stream
  *    with no encode in between, so the tile index and ticket are still zero and
@@ -136,6 +139,8 @@ int cszp2_compress_prepare_range(const void *d_in, uint64_t n, int dtype, double
 #define CSZP2_FLAG_LOAD_VEC 2u
 #define CSZP2_FLAG_LOAD_SCALAR 4u
 #define CSZP2_FLAG_PREPARED 8u
+#define CSZP2_FLAG_LB_WIDE 16u
+#define CSZP2_FLAG_LB_NARROW 32u
 int cszp2_compress_encode_ex(const void *d_in, uint64_t n, int dtype, double eb, int eb_mode,
                              int enc_mode, void *d_out, uint64_t *d_out_bytes, unsigned flags,
                              void *stream);

@@ -175,12 +175,12 @@ int launch_minmax(const void *d_in, uint64_t n, double lambda, void *d_out, cuda
     return launch_status();
 }
 
-template <typename T, bool OUTLIER, int LOAD>
+template <typename T, bool OUTLIER, int LOAD, int LBR = LB_PER_LANE>
 int launch_compress_l(const void *d_in, const Geom &g, double eb, int eb_mode, int enc_mode,
                       void *d_out, uint64_t *d_out_bytes, cudaStream_t st, unsigned flags) {
     constexpr int smem = compress_smem_bytes<T>();
-    if (int rc = set_smem(compress_kernel<T, OUTLIER, LOAD>, smem)) return rc;
-    const unsigned grid = persistent_grid(compress_kernel<T, OUTLIER, LOAD>, NT_COMP, smem, g.T);
+    if (int rc = set_smem(compress_kernel<T, OUTLIER, LOAD, LBR>, smem)) return rc;
+    const unsigned grid = persistent_grid(compress_kernel<T, OUTLIER, LOAD, LBR>, NT_COMP, smem, g.T);
     unsigned *ticket = reinterpret_cast<unsigned *>(static_cast<uint8_t *>(d_out) + stream_bound(g));
     // the lookback descriptors (= the tile index, and its pad to O) and the tile ticket
     // start from zero on every encode, so encode can be repeated on one buffer
@@ -196,7 +196,7 @@ int launch_compress_l(const void *d_in, const Geom &g, double eb, int eb_mode, i
     hs.eb_mode = static_cast<uint32_t>(eb_mode);
     hs.eb_user = eb;
     hs.flags = flags;
-    compress_kernel<T, OUTLIER, LOAD><<<grid, NT_COMP, smem, st>>>(
+    compress_kernel<T, OUTLIER, LOAD, LBR><<<grid, NT_COMP, smem, st>>>(
         map, static_cast<const T *>(d_in), g, eb, eb_mode == CSZP2_EB_REL ? 1 : 0,
         static_cast<uint8_t *>(d_out), ticket, d_out_bytes, hs);
     return launch_status();
@@ -209,6 +209,10 @@ int launch_compress(const void *d_in, const Geom &g, double eb, int eb_mode, int
         return launch_compress_l<T, OUTLIER, LOAD_VEC>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags);
     if (flags & CSZP2_FLAG_LOAD_SCALAR)
         return launch_compress_l<T, OUTLIER, LOAD_SCALAR>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags);
+    // lookback window: 32 wide up to LB_NARROW_TILES tiles, 256 wide beyond (kernels.cuh)
+    const bool narrow = (flags & CSZP2_FLAG_LB_NARROW) || (!(flags & CSZP2_FLAG_LB_WIDE) && g.T <= LB_NARROW_TILES);
+    if (narrow)
+        return launch_compress_l<T, OUTLIER, LOAD_TMA, 1>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags);
     return launch_compress_l<T, OUTLIER, LOAD_TMA>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags);
 }
 
@@ -265,13 +269,13 @@ void nd_rows(GeomND &g) {
     g.vec = (g.nx % (16 / sizeof(T))) == 0 ? 1u : 0u;
 }
 
-template <typename T, int NDIM, bool OUTLIER>
-int launch_compress_nd(const void *d_in, const GeomND &g0, double eb, int eb_mode, int enc_mode,
-                       void *d_out, uint64_t *d_out_bytes, cudaStream_t st) {
+template <typename T, int NDIM, bool OUTLIER, int LBR>
+int launch_compress_nd_w(const void *d_in, const GeomND &g0, double eb, int eb_mode, int enc_mode,
+                         void *d_out, uint64_t *d_out_bytes, cudaStream_t st) {
     constexpr int smem = ND_RING + 64;
     GeomND g = g0;  // + the gather strides of this value type
     nd_rows<T, NDIM>(g);
-    if (int rc = set_smem(compress_nd_kernel<T, NDIM, OUTLIER>, smem)) return rc;
+    if (int rc = set_smem(compress_nd_kernel<T, NDIM, OUTLIER, LBR>, smem)) return rc;
     unsigned *ticket = reinterpret_cast<unsigned *>(static_cast<uint8_t *>(d_out) + stream_bound_nd(g));
     HdrStatic hs;
     hs.word1 = 1u | (static_cast<uint32_t>(Traits<T>::DTYPE) << 8) |
@@ -279,11 +283,19 @@ int launch_compress_nd(const void *d_in, const GeomND &g0, double eb, int eb_mod
     hs.eb_mode = static_cast<uint32_t>(eb_mode);
     hs.eb_user = eb;
     hs.flags = 0;
-    const unsigned grid = persistent_grid(compress_nd_kernel<T, NDIM, OUTLIER>, NT_COMP, smem, g.T);
-    compress_nd_kernel<T, NDIM, OUTLIER><<<grid, NT_COMP, smem, st>>>(
+    const unsigned grid = persistent_grid(compress_nd_kernel<T, NDIM, OUTLIER, LBR>, NT_COMP, smem, g.T);
+    compress_nd_kernel<T, NDIM, OUTLIER, LBR><<<grid, NT_COMP, smem, st>>>(
         static_cast<const T *>(d_in), g, eb, eb_mode == CSZP2_EB_REL ? 1 : 0,
         static_cast<uint8_t *>(d_out), ticket, d_out_bytes, hs);
     return launch_status();
+}
+template <typename T, int NDIM, bool OUTLIER>
+int launch_compress_nd(const void *d_in, const GeomND &g, double eb, int eb_mode, int enc_mode,
+                       void *d_out, uint64_t *d_out_bytes, cudaStream_t st) {
+    // lookback window: 32 wide up to LB_NARROW_TILES tiles, 256 wide beyond (kernels.cuh)
+    if (g.T <= LB_NARROW_TILES)
+        return launch_compress_nd_w<T, NDIM, OUTLIER, 1>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st);
+    return launch_compress_nd_w<T, NDIM, OUTLIER, LB_PER_LANE>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st);
 }
 
 template <typename T, int NDIM>
@@ -375,9 +387,11 @@ int cszp2_compress_encode_ex(const void *d_in, uint64_t n, int dtype, double eb,
     int rc = check_compress_args(d_in, n, dtype, eb, eb_mode, d_out);
     if (rc) return rc;
     if (enc_mode != CSZP2_ENC_PLAIN && enc_mode != CSZP2_ENC_OUTLIER) return CSZP2_ERR_ARG;
-    if (flags & ~(CSZP2_FLAG_CHAINED_SCAN | CSZP2_FLAG_LOAD_VEC | CSZP2_FLAG_LOAD_SCALAR | CSZP2_FLAG_PREPARED))
+    if (flags & ~(CSZP2_FLAG_CHAINED_SCAN | CSZP2_FLAG_LOAD_VEC | CSZP2_FLAG_LOAD_SCALAR | CSZP2_FLAG_PREPARED |
+                  CSZP2_FLAG_LB_WIDE | CSZP2_FLAG_LB_NARROW))
         return CSZP2_ERR_ARG;
     if ((flags & CSZP2_FLAG_LOAD_VEC) && (flags & CSZP2_FLAG_LOAD_SCALAR)) return CSZP2_ERR_ARG;
+    if ((flags & CSZP2_FLAG_LB_WIDE) && (flags & CSZP2_FLAG_LB_NARROW)) return CSZP2_ERR_ARG;
     Geom g = geometry(n);
     cudaStream_t st = S(stream);
     if (dtype == CSZP2_F32)

@@ -475,16 +475,18 @@ __device__ __forceinline__ void publish_aggregate(uint64_t *index, uint64_t t, u
     st_relaxed_u64(&index[t], (t == 0 ? FLAG_P : FLAG_A) | (bad ? BIT_RANGE : 0) | agg);
 }
 
+template <int ROWS = LB_PER_LANE>
 struct LookbackWindow {
-    uint64_t d[LB_PER_LANE];
+    uint64_t d[ROWS];
 };
 
 // Window rows: row u, lane l holds the descriptor of tile j − (32u + l) (nearest first;
 // each row is one coalesced 256-byte load).
-__device__ __forceinline__ void lookback_issue(const uint64_t *index, int64_t j, LookbackWindow &w) {
+template <int ROWS>
+__device__ __forceinline__ void lookback_issue(const uint64_t *index, int64_t j, LookbackWindow<ROWS> &w) {
     const int64_t base = j - (threadIdx.x & 31);
 #pragma unroll
-    for (int u = 0; u < LB_PER_LANE; u++)
+    for (int u = 0; u < ROWS; u++)
         w.d[u] = (base - 32 * u >= 0) ? ld_relaxed_u64(&index[base - 32 * u]) : FLAG_P;  // virtual P|0
 }
 
@@ -495,8 +497,9 @@ __device__ __forceinline__ void lookback_issue(const uint64_t *index, int64_t j,
 // reductions; if a Waiting slot is nearer than the P, the Waiting slots are re-polled;
 // otherwise every slot before the P is an A, whose values (tile aggregates, each
 // <= 256 * 132 bytes, so 256 of them fit in 32 bits) are summed by one reduction.
+template <int ROWS>
 __device__ __forceinline__ uint64_t lookback_finish(uint64_t *index, uint64_t t, uint64_t agg,
-                                                    bool bad, LookbackWindow &w, bool *range_out) {
+                                                    bool bad, LookbackWindow<ROWS> &w, bool *range_out) {
     const int lane = threadIdx.x & 31;
     uint64_t excl = 0;
     bool rb = bad;
@@ -504,7 +507,7 @@ __device__ __forceinline__ uint64_t lookback_finish(uint64_t *index, uint64_t t,
     while (true) {
         uint32_t pk = 0xFFFFu, wk = 0xFFFFu;
 #pragma unroll
-        for (int u = LB_PER_LANE - 1; u >= 0; u--) {  // descending: the nearest row wins
+        for (int u = ROWS - 1; u >= 0; u--) {  // descending: the nearest row wins
             const uint32_t f = static_cast<uint32_t>(w.d[u] >> 62);
             if (f == 2) pk = 32u * u + lane;
             if (f == 0) wk = 32u * u + lane;
@@ -524,7 +527,7 @@ __device__ __forceinline__ uint64_t lookback_finish(uint64_t *index, uint64_t t,
 #endif
             __nanosleep(32);
 #pragma unroll
-            for (int u = 0; u < LB_PER_LANE; u++) {
+            for (int u = 0; u < ROWS; u++) {
                 const int64_t idx = j - 32 * u - lane;
                 if ((w.d[u] >> 62) == 0 && idx >= 0) w.d[u] = ld_relaxed_u64(&index[idx]);
             }
@@ -534,7 +537,7 @@ __device__ __forceinline__ uint64_t lookback_finish(uint64_t *index, uint64_t t,
         bool r = false;
         uint64_t pv = 0;
 #pragma unroll
-        for (int u = 0; u < LB_PER_LANE; u++) {
+        for (int u = 0; u < ROWS; u++) {
             const uint32_t key = 32u * u + lane;
             const uint64_t d = w.d[u];
             if (key < P) s += static_cast<uint32_t>(d);  // an A: value < 2^32
@@ -543,14 +546,14 @@ __device__ __forceinline__ uint64_t lookback_finish(uint64_t *index, uint64_t t,
         }
         excl += __reduce_add_sync(0xffffffffu, s);
         rb |= __any_sync(0xffffffffu, r);
-        if (P < 32u * LB_PER_LANE) {
+        if (P < 32u * ROWS) {
             excl += __shfl_sync(0xffffffffu, pv, P & 31u);
             break;
         }
 #ifdef CSZP2_TRACE
         if (lane == 0 && g_trace) g_trace[t * 16 + 5] += 1ll << 32;  // extra window
 #endif
-        j -= 32 * LB_PER_LANE;
+        j -= 32 * ROWS;
         lookback_issue(index, j, w);
     }
     if (lane == 0) st_relaxed_u64(&index[t], FLAG_P | (rb ? BIT_RANGE : 0) | (excl + agg));
@@ -558,13 +561,21 @@ __device__ __forceinline__ uint64_t lookback_finish(uint64_t *index, uint64_t t,
     return excl;
 }
 
-// Issue the first window and resolve (used by the compression consumer warp).
+// Issue the first window and resolve (used by the compression consumer warp). Window
+// width 32 x ROWS: the compressors are instantiated with 256 (ROWS = 8) for fields of
+// more than LB_NARROW_TILES tiles and 32 (ROWS = 1, windows walked one row at a time)
+// for smaller ones (chosen at launch) — measured, not derived: on configs 2-4b (≤ 34k tiles) the 32-wide window is
+// 3-10% faster (1D configs 3a/4a, the 3D kernel), on config 5 (2^20 tiles) 8-10% slower
+// (profiles/ab_lookback_window_r02b.txt).
+constexpr uint64_t LB_NARROW_TILES = 1ull << 17;
+template <int ROWS = LB_PER_LANE>
 __device__ __forceinline__ uint64_t lookback(uint64_t *index, uint64_t t, uint64_t agg, bool bad,
                                              bool *range_out) {
-    LookbackWindow w;
-    lookback_issue(index, static_cast<int64_t>(t) - 1, w);
-    return lookback_finish(index, t, agg, bad, w, range_out);
+    LookbackWindow<ROWS> w;
+    lookback_issue<ROWS>(index, static_cast<int64_t>(t) - 1, w);
+    return lookback_finish<ROWS>(index, t, agg, bad, w, range_out);
 }
+
 
 // Ablation (NEXT #2): the plain chained scan that decoupled lookback replaces
 // (Fig 12 left) — wait until the immediate predecessor holds its
@@ -890,7 +901,7 @@ __device__ __forceinline__ void write_payload(const uint8_t *stg, uint8_t *out, 
 // paper's vectorised access), 2 = each thread reads its block value by value.
 constexpr int LOAD_TMA = 0, LOAD_VEC = 1, LOAD_SCALAR = 2;
 
-template <typename T, bool OUTLIER, int LOAD = LOAD_TMA>
+template <typename T, bool OUTLIER, int LOAD = LOAD_TMA, int LBR = LB_PER_LANE>
 __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kernel(
     const __grid_constant__ CUtensorMap tmap, const T *__restrict__ in, const Geom g,
     const double eb_abs_arg, const int eb_from_header, uint8_t *__restrict__ out,
@@ -1197,7 +1208,7 @@ __global__ void __launch_bounds__(NT_COMP, sizeof(T) == 4 ? 3 : 2) compress_kern
                 if (chained)  // ablation: plain chained scan (Fig 12 left)
                     excl = chained_prefix(index, t, agg, bad, &rng);
                 else
-                    excl = lookback(index, t, agg, bad, &rng);
+                    excl = lookback<LBR>(index, t, agg, bad, &rng);
             }
             if (lane == 0) TRACE(t, 3, gtimer());
             const uint64_t dst0 = g.D + excl;

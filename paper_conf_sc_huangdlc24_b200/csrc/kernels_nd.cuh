@@ -321,7 +321,7 @@ constexpr uint32_t ND_RING = 96 * 1024;              // compression staging ring
 // barrier waits on a lookback (round 1 ran it in warp 0 between two __syncthreads).
 constexpr uint32_t ND_RING_V = 128 * 1024;  // virtual lap of the ring (a power of 2 >= ND_RING)
 
-template <typename T, int NDIM, bool OUTLIER>
+template <typename T, int NDIM, bool OUTLIER, int LBR = LB_PER_LANE>
 __global__ void __launch_bounds__(NT_COMP, 2) compress_nd_kernel(const T *__restrict__ in, const GeomND g,
                                                                  const double eb_abs_arg,
                                                                  const int eb_from_header,
@@ -545,7 +545,7 @@ __global__ void __launch_bounds__(NT_COMP, 2) compress_nd_kernel(const T *__rest
             const bool bad = s_qbad[q];
             bool rng = bad;
             uint64_t excl = 0;
-            if (g.T && t > 0) excl = lookback(index, t, agg, bad, &rng);
+            if (g.T && t > 0) excl = lookback<LBR>(index, t, agg, bad, &rng);
             const uint64_t dst0 = g.D + excl;
             write_payload(ring + (pos % ND_RING_V), out, dst0, agg, lane, 32);
             if (t == T_eff - 1) {  // last tile: pads, header, d_out_bytes

@@ -438,7 +438,7 @@ def test_c_abi_rejects_invalid_arguments():
     assert L.cszp2_compress(p(x, 4), 10, 0, 1e-3, 0, 0, p(out), p(nb), s) == E       # misaligned in
     assert L.cszp2_compress(p(x), 10, 0, 1e-3, 0, 0, p(out, 8), p(nb), s) == E       # misaligned out
     assert L.cszp2_compress(p(x), (1 << 35) + 1, 0, 1e-3, 0, 0, p(out), p(nb), s) == E  # n too large
-    assert L.cszp2_compress_encode_ex(p(x), 10, 0, 1e-3, 0, 0, p(out), p(nb), 16, s) == E  # flags
+    assert L.cszp2_compress_encode_ex(p(x), 10, 0, 1e-3, 0, 0, p(out), p(nb), 64, s) == E  # flags
     assert L.cszp2_compress_encode_ex(p(x), 10, 0, 1e-3, 0, 0, p(out), p(nb), 6, s) == E  # vec+scalar
     assert L.cszp2_decompress(None, p(x), 10, 0, None, s) == E
     assert L.cszp2_decompress(p(out), p(x, 4), 10, 0, None, s) == E
@@ -558,3 +558,27 @@ def test_repeated_runs_are_deterministic(cfg, enc):
     ref, rc = oracle.compress(x.cpu().numpy(), lam, EBM[spec.eb_mode], ENC[enc])
     assert rc == oracle.OK
     np.testing.assert_array_equal(first.cpu().numpy(), ref)
+
+
+@pytest.mark.parametrize("flags", [16, 32])
+@pytest.mark.parametrize("enc", ["plain", "outlier"])
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_lookback_window_width_same_stream(flags, enc, dtype):
+    """The lookback's first window is 32 predecessors up to 2^17 tiles and 256 beyond (a
+    speed choice, kernels.cuh LB_NARROW_TILES); forcing either width (FLAG_LB_WIDE /
+    FLAG_LB_NARROW) on a field of ~1700 tiles — several per CTA, lookbacks across many
+    windows — gives the oracle's stream byte for byte."""
+    n = 1700 * 8192 + 32 * 5 + 9
+    xh = make_field("cfg4a", DEV, 0, n).cpu().numpy().astype(dtype)
+    x = torch.from_numpy(xh).to(DEV)
+    ref, rc = oracle.compress(xh, 1e-4, oracle.REL, oracle.OUTLIER if enc == "outlier" else oracle.PLAIN)
+    assert rc == oracle.OK
+    out = torch.full((cz.compress_bound(n, x.dtype),), 0xAA, dtype=torch.uint8, device=DEV)
+    nb = torch.zeros(1, dtype=torch.int64, device=DEV)
+    cz.compress_prepare(x, 1e-4, "rel", out)
+    cz.compress_encode_ex(x, 1e-4, "rel", enc, out, nb, flags=flags)
+    torch.cuda.synchronize()
+    assert int(nb.item()) == ref.size
+    np.testing.assert_array_equal(out[: ref.size].cpu().numpy(), ref)
+    with pytest.raises(cz.CszpError):
+        cz.compress_encode_ex(x, 1e-4, "rel", enc, out, nb, flags=48)
