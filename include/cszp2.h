@@ -226,12 +226,18 @@ int cszp2_container_index(const uint64_t *d_sizes, int nparts, uint64_t *d_offse
  * cszp2_compress_nd: like cszp2_compress (same eb / eb_mode / enc_mode meaning,
  *   same RANGE behaviour with this predictor's tighter limit |x/2eb| <= 2^28-1 (2D)
  *   or 2^27-1 (3D), FORMAT.md §7); asynchronous on `stream`.
+ * cszp2_compress_nd_ex: the same with flags: CSZP2_FLAG_LB_WIDE / CSZP2_FLAG_LB_NARROW
+ *   as for cszp2_compress_encode_ex (same stream bytes either way); any other bit, or
+ *   both, is ARG.
  * cszp2_decompress_nd: inverse; d_out = nx*ny*nz values, device, 16-byte aligned;
  *   d_status as in cszp2_decompress. */
 uint64_t cszp2_compress_bound_nd(uint64_t nx, uint64_t ny, uint64_t nz, int ndim, int dtype);
 int cszp2_compress_nd(const void *d_in, uint64_t nx, uint64_t ny, uint64_t nz, int ndim, int dtype,
                       double eb, int eb_mode, int enc_mode, void *d_out, uint64_t *d_out_bytes,
                       void *stream);
+int cszp2_compress_nd_ex(const void *d_in, uint64_t nx, uint64_t ny, uint64_t nz, int ndim, int dtype,
+                         double eb, int eb_mode, int enc_mode, void *d_out, uint64_t *d_out_bytes,
+                         unsigned flags, void *stream);
 int cszp2_decompress_nd(const void *d_cmp, void *d_out, uint64_t nx, uint64_t ny, uint64_t nz, int ndim,
                         int dtype, int *d_status, void *stream);
 

@@ -79,6 +79,7 @@ def _load():
     L.cszp2_compress_bound_nd.argtypes = [u64, u64, u64, i32, i32]
     L.cszp2_compress_bound_nd.restype = u64
     L.cszp2_compress_nd.argtypes = [vp, u64, u64, u64, i32, i32, dbl, i32, i32, vp, vp, vp]
+    L.cszp2_compress_nd_ex.argtypes = [vp, u64, u64, u64, i32, i32, dbl, i32, i32, vp, vp, ctypes.c_uint, vp]
     L.cszp2_decompress_nd.argtypes = [vp, vp, u64, u64, u64, i32, i32, vp, vp]
     L.cszp2_version.restype = ctypes.c_char_p
     return L
@@ -91,7 +92,7 @@ EXPORTED = (
     "cszp2_compress_encode_ex", "cszp2_value_range", "cszp2_compress_prepare_range",
     "cszp2_decompress", "cszp2_decompress_range", "cszp2_read_header", "cszp2_compress_host", "cszp2_decompress_host",
     "cszp2_container_index", "cszp2_version",
-    "cszp2_compress_bound_nd", "cszp2_compress_nd", "cszp2_decompress_nd",
+    "cszp2_compress_bound_nd", "cszp2_compress_nd", "cszp2_compress_nd_ex", "cszp2_decompress_nd",
     "cszp2_decompress_scratch_bytes", "cszp2_decompress_tilewise",
 )
 
@@ -397,9 +398,10 @@ def compress_bound_nd(shape, dtype=torch.float32) -> int:
 
 
 def compress_nd(x: torch.Tensor, eb: float, eb_mode="abs", enc_mode="outlier", out=None, out_bytes=None,
-                stream=None):
+                stream=None, flags=0):
     """2D (8x8 blocks) / 3D (4x4x4 blocks) Lorenzo compression of a 2D/3D CUDA
-    tensor (last axis fastest; FORMAT.md §7). Returns (buffer, device byte count)."""
+    tensor (last axis fastest; FORMAT.md §7). Returns (buffer, device byte count).
+    flags: FLAG_LB_WIDE / FLAG_LB_NARROW force the lookback window (same stream)."""
     dev = _need_cuda(x, out, out_bytes)
     x = x.contiguous()
     nx, ny, nz, nd = _extents(x.shape)
@@ -412,8 +414,8 @@ def compress_nd(x: torch.Tensor, eb: float, eb_mode="abs", enc_mode="outlier", o
         raise ValueError("out must be a contiguous uint8 tensor of compress_bound_nd bytes")
     _need_word(out_bytes, (torch.int64, torch.uint64), "out_bytes")
     with torch.cuda.device(dev):
-        rc = _lib.cszp2_compress_nd(_ptr(x), nx, ny, nz, nd, dt, float(eb), _EB[eb_mode], _ENC[enc_mode],
-                                    _ptr(out), _ptr(out_bytes), _stream(stream))
+        rc = _lib.cszp2_compress_nd_ex(_ptr(x), nx, ny, nz, nd, dt, float(eb), _EB[eb_mode], _ENC[enc_mode],
+                                       _ptr(out), _ptr(out_bytes), int(flags), _stream(stream))
     _check("cszp2_compress_nd", rc)
     return out, out_bytes
 

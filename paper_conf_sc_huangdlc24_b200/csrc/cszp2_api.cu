@@ -291,9 +291,10 @@ int launch_compress_nd_w(const void *d_in, const GeomND &g0, double eb, int eb_m
 }
 template <typename T, int NDIM, bool OUTLIER>
 int launch_compress_nd(const void *d_in, const GeomND &g, double eb, int eb_mode, int enc_mode,
-                       void *d_out, uint64_t *d_out_bytes, cudaStream_t st) {
-    // lookback window: 32 wide up to LB_NARROW_TILES tiles, 256 wide beyond (kernels.cuh)
-    if (g.T <= LB_NARROW_TILES)
+                       void *d_out, uint64_t *d_out_bytes, cudaStream_t st, unsigned flags) {
+    // lookback window: 32 wide up to LB_NARROW_TILES tiles, 256 wide beyond (kernels.cuh),
+    // unless forced by CSZP2_FLAG_LB_NARROW / CSZP2_FLAG_LB_WIDE
+    if ((flags & CSZP2_FLAG_LB_NARROW) || (!(flags & CSZP2_FLAG_LB_WIDE) && g.T <= LB_NARROW_TILES))
         return launch_compress_nd_w<T, NDIM, OUTLIER, 1>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st);
     return launch_compress_nd_w<T, NDIM, OUTLIER, LB_PER_LANE>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st);
 }
@@ -322,13 +323,13 @@ int launch_decompress_nd(const void *d_cmp, void *d_out, const GeomND &g0, int *
 
 template <typename T>
 int dispatch_compress_nd(const void *d_in, const GeomND &g, int ndim, double eb, int eb_mode,
-                         int enc_mode, void *d_out, uint64_t *d_out_bytes, cudaStream_t st) {
+                         int enc_mode, void *d_out, uint64_t *d_out_bytes, cudaStream_t st, unsigned flags) {
     const bool o = enc_mode == CSZP2_ENC_OUTLIER;
     if (ndim == 2)
-        return o ? launch_compress_nd<T, 2, true>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st)
-                 : launch_compress_nd<T, 2, false>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st);
-    return o ? launch_compress_nd<T, 3, true>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st)
-             : launch_compress_nd<T, 3, false>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st);
+        return o ? launch_compress_nd<T, 2, true>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags)
+                 : launch_compress_nd<T, 2, false>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags);
+    return o ? launch_compress_nd<T, 3, true>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags)
+             : launch_compress_nd<T, 3, false>(d_in, g, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags);
 }
 
 }  // namespace
@@ -551,7 +552,16 @@ uint64_t cszp2_compress_bound_nd(uint64_t nx, uint64_t ny, uint64_t nz, int ndim
 int cszp2_compress_nd(const void *d_in, uint64_t nx, uint64_t ny, uint64_t nz, int ndim, int dtype,
                       double eb, int eb_mode, int enc_mode, void *d_out, uint64_t *d_out_bytes,
                       void *stream) {
+    return cszp2_compress_nd_ex(d_in, nx, ny, nz, ndim, dtype, eb, eb_mode, enc_mode, d_out, d_out_bytes, 0u,
+                                stream);
+}
+
+int cszp2_compress_nd_ex(const void *d_in, uint64_t nx, uint64_t ny, uint64_t nz, int ndim, int dtype,
+                         double eb, int eb_mode, int enc_mode, void *d_out, uint64_t *d_out_bytes,
+                         unsigned flags, void *stream) {
     GeomND g;
+    if (flags & ~(CSZP2_FLAG_LB_WIDE | CSZP2_FLAG_LB_NARROW)) return CSZP2_ERR_ARG;
+    if ((flags & CSZP2_FLAG_LB_WIDE) && (flags & CSZP2_FLAG_LB_NARROW)) return CSZP2_ERR_ARG;
     if (geometry_nd(nx, ny, nz, ndim, &g)) return CSZP2_ERR_ARG;
     if (enc_mode != CSZP2_ENC_PLAIN && enc_mode != CSZP2_ENC_OUTLIER) return CSZP2_ERR_ARG;
     int rc = check_compress_args(d_in, g.n, dtype, eb, eb_mode, d_out);
@@ -566,8 +576,8 @@ int cszp2_compress_nd(const void *d_in, uint64_t nx, uint64_t ny, uint64_t nz, i
         if (rc) return rc;
     }
     return dtype == CSZP2_F32
-               ? dispatch_compress_nd<float>(d_in, g, ndim, eb, eb_mode, enc_mode, d_out, d_out_bytes, st)
-               : dispatch_compress_nd<double>(d_in, g, ndim, eb, eb_mode, enc_mode, d_out, d_out_bytes, st);
+               ? dispatch_compress_nd<float>(d_in, g, ndim, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags)
+               : dispatch_compress_nd<double>(d_in, g, ndim, eb, eb_mode, enc_mode, d_out, d_out_bytes, st, flags);
 }
 
 int cszp2_decompress_nd(const void *d_cmp, void *d_out, uint64_t nx, uint64_t ny, uint64_t nz, int ndim,

@@ -228,3 +228,24 @@ def test_nd_decompress_rejects_corrupt_streams(dtype):
         bad = out.clone()
         bad[64 + 8 * t + 7] = 0  # descriptor flag cleared
         assert status(bad) == 4
+
+
+@pytest.mark.parametrize("flags", [cz.FLAG_LB_WIDE, cz.FLAG_LB_NARROW])
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_nd_lookback_window_width_same_stream(flags, dtype):
+    """The nD compressor is instantiated for 32- and 256-wide first lookback windows
+    (32 up to 2^17 tiles, kernels.cuh); forcing either on a 1024-tile field gives the
+    oracle's stream, so the 256-wide one is covered without an 8 GiB field."""
+    shape = (256, 256, 256)
+    xh = smooth_field(shape, 13, dtype, noise=1e-2)
+    x = torch.from_numpy(xh).to(DEV)
+    ref, rc = oracle.compress_nd(xh, 1e-4, oracle.REL, oracle.OUTLIER)
+    assert rc == oracle.OK
+    out = torch.full((cz.compress_bound_nd(xh.shape, x.dtype),), 0xAA, dtype=torch.uint8, device=DEV)
+    nb = torch.zeros(1, dtype=torch.int64, device=DEV)
+    cz.compress_nd(x, 1e-4, "rel", "outlier", out=out, out_bytes=nb, flags=flags)
+    torch.cuda.synchronize()
+    assert int(nb.item()) == ref.size
+    np.testing.assert_array_equal(out[: ref.size].cpu().numpy(), ref)
+    with pytest.raises(cz.CszpError):
+        cz.compress_nd(x, 1e-4, "rel", "outlier", out=out, out_bytes=nb, flags=cz.FLAG_LB_WIDE | cz.FLAG_LB_NARROW)
