@@ -128,7 +128,7 @@ int cszp2_compress_prepare_range(const void *d_in, uint64_t n, int dtype, double
  *    non-vectorised baseline of the §VI-E memory ablation).
  *  LOAD_VEC and LOAD_SCALAR are exclusive (ARG otherwise).
  *  CSZP2_FLAG_LB_WIDE / CSZP2_FLAG_LB_NARROW: force the lookback's first window
- *    to 256 / 32 predecessors (by default 32 up to 2^17 tiles, 256 beyond; a speed
+ *    to 256 / 32 predecessors (by default 32 below 2^16 tiles, 256 from 2^16 on; a speed
  *    choice that changes no stream byte). Exclusive (ARG otherwise).
  *  CSZP2_FLAG_PREPARED (not an ablation): the caller guarantees that a
  *    cszp2_compress_prepare(_range) on this d_out precedes this call on the stream

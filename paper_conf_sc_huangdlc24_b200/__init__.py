@@ -242,7 +242,7 @@ FLAG_CHAINED_SCAN = 1
 FLAG_LOAD_VEC = 2
 FLAG_LOAD_SCALAR = 4
 FLAG_PREPARED = 8  # a prepare on this buffer precedes the encode: skip re-zeroing (include/cszp2.h)
-FLAG_LB_WIDE = 16  # lookback first window 256 / 32 predecessors (default: by tile count)
+FLAG_LB_WIDE = 16  # lookback first window 256 / 32 predecessors (default: by tile count, 32 below 2^16 tiles)
 FLAG_LB_NARROW = 32
 
 

@@ -562,12 +562,13 @@ __device__ __forceinline__ uint64_t lookback_finish(uint64_t *index, uint64_t t,
 }
 
 // Issue the first window and resolve (used by the compression consumer warp). Window
-// width 32 x ROWS: the compressors are instantiated with 256 (ROWS = 8) for fields of
-// more than LB_NARROW_TILES tiles and 32 (ROWS = 1, windows walked one row at a time)
-// for smaller ones (chosen at launch) — measured, not derived: on configs 2-4b (≤ 34k tiles) the 32-wide window is
-// 3-10% faster (1D configs 3a/4a, the 3D kernel), on config 5 (2^20 tiles) 8-10% slower
-// (profiles/ab_lookback_window_r02b.txt).
-constexpr uint64_t LB_NARROW_TILES = 1ull << 17;
+// width 32 x ROWS: the compressors are instantiated with 256 (ROWS = 8) and with 32
+// (ROWS = 1, windows walked one row at a time); the launch takes 32 for fields of at
+// most LB_NARROW_TILES tiles. Measured, not derived: on configs 2-4b (≤ 34k tiles) the
+// 32-wide window is 3-10% faster (1D configs 3a/4a, the 3D kernel); on config 5's data it
+// ties at 2^15 tiles and loses from 2^16 tiles on (4-8% at 2^17, a config 5 slab at 8 GPUs;
+// 8-10% at 2^20) (profiles/ab_lookback_window_r02b.txt).
+constexpr uint64_t LB_NARROW_TILES = (1ull << 16) - 1;
 template <int ROWS = LB_PER_LANE>
 __device__ __forceinline__ uint64_t lookback(uint64_t *index, uint64_t t, uint64_t agg, bool bad,
                                              bool *range_out) {

@@ -234,7 +234,7 @@ def test_nd_decompress_rejects_corrupt_streams(dtype):
 @pytest.mark.parametrize("dtype", [np.float32, np.float64])
 def test_nd_lookback_window_width_same_stream(flags, dtype):
     """The nD compressor is instantiated for 32- and 256-wide first lookback windows
-    (32 up to 2^17 tiles, kernels.cuh); forcing either on a 1024-tile field gives the
+    (32 below 2^16 tiles, kernels.cuh); forcing either on a 1024-tile field gives the
     oracle's stream, so the 256-wide one is covered without an 8 GiB field."""
     shape = (256, 256, 256)
     xh = smooth_field(shape, 13, dtype, noise=1e-2)

@@ -564,7 +564,7 @@ def test_repeated_runs_are_deterministic(cfg, enc):
 @pytest.mark.parametrize("enc", ["plain", "outlier"])
 @pytest.mark.parametrize("dtype", [np.float32, np.float64])
 def test_lookback_window_width_same_stream(flags, enc, dtype):
-    """The lookback's first window is 32 predecessors up to 2^17 tiles and 256 beyond (a
+    """The lookback's first window is 32 predecessors below 2^16 tiles and 256 from there on (a
     speed choice, kernels.cuh LB_NARROW_TILES); forcing either width (FLAG_LB_WIDE /
     FLAG_LB_NARROW) on a field of ~1700 tiles — several per CTA, lookbacks across many
     windows — gives the oracle's stream byte for byte."""
