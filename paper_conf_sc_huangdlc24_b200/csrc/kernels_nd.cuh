@@ -58,20 +58,6 @@ struct BlockShape<3> {
     static constexpr int BX = 4, BY = 4, BZ = 4;
 };
 
-// FORMAT.md §7 range limits: |d| <= 2^ndim * max|q| must fit the 31-bit code
-template <int NDIM>
-__device__ __forceinline__ int quantize_nd(float x, float inv, bool &bad) {
-    const float t = __fmul_rn(x, inv);
-    bad |= !(fabsf(t) <= (NDIM == 2 ? 268435440.0f : 134217720.0f));
-    return __float2int_rn(t);
-}
-template <int NDIM>
-__device__ __forceinline__ int quantize_nd(double x, double inv, bool &bad) {
-    const double t = __dmul_rn(x, inv);
-    bad |= !(fabs(t) <= (NDIM == 2 ? 268435455.0 : 134217727.0));
-    return __double2int_rn(t);
-}
-
 // Lorenzo prediction of in-block value i from its lower neighbours (block-local:
 // neighbours outside the block are 0), "3 and 7 adjacent data points".
 template <int NDIM>
@@ -136,7 +122,8 @@ __device__ __forceinline__ bool interior_vec(const GeomND &g, const BlockOrigin 
 
 // ❶ for one value, as a BIASED pattern (f32: q + 0x4B400000 mod 2^32; f64: q).
 // UNCHECKED (f32 only): the bits of fl(x·inv + 1.5·2^23), exact whenever the block passes
-// the certificate in compress_nd_kernel; CHECKED: FORMAT.md §7's range check.
+// the certificate in compress_nd_kernel; CHECKED: FORMAT.md §7's range check (|d| <=
+// 2^ndim · max|q| must fit the 31-bit code: |x/2eb| <= 2^28-1 in 2D, 2^27-1 in 3D).
 template <int NDIM, bool CHECKED>
 __device__ __forceinline__ uint32_t qpattern(float x, float inv, bool &bad) {
     const float t = __fmul_rn(x, inv);
