@@ -267,6 +267,7 @@ void nd_rows(GeomND &g) {
     g.ystep = g.roff[1];
     g.zstep = NDIM == 3 ? g.roff[4] - g.roff[3] : 0;
     g.vec = (g.nx % (16 / sizeof(T))) == 0 ? 1u : 0u;
+    g.vec32 = 0;  // set by the launch from the buffer it accesses
 }
 
 template <typename T, int NDIM, bool OUTLIER, int LBR>
@@ -275,6 +276,7 @@ int launch_compress_nd_w(const void *d_in, const GeomND &g0, double eb, int eb_m
     constexpr int smem = ND_RING + 64;
     GeomND g = g0;  // + the gather strides of this value type
     nd_rows<T, NDIM>(g);
+    g.vec32 = (reinterpret_cast<uintptr_t>(d_in) % 32 == 0 && (g.nx * sizeof(T)) % 32 == 0) ? 1u : 0u;
     if (int rc = set_smem(compress_nd_kernel<T, NDIM, OUTLIER, LBR>, smem)) return rc;
     unsigned *ticket = reinterpret_cast<unsigned *>(static_cast<uint8_t *>(d_out) + stream_bound_nd(g));
     HdrStatic hs;
@@ -305,15 +307,18 @@ int launch_decompress_nd(const void *d_cmp, void *d_out, const GeomND &g0, int *
     if constexpr (sizeof(T) == 8) {  // f64: one CTA per tile (kernels_nd.cuh, decompress_nd_tile_kernel)
         constexpr int smem = ND_STAGE + 64;
         if (int rc = set_smem(decompress_nd_tile_kernel<T, NDIM>, smem)) return rc;
-        const unsigned grid = static_cast<unsigned>(g0.T ? g0.T : 1);
+        GeomND g = g0;
+        g.vec32 = (reinterpret_cast<uintptr_t>(d_out) % 32 == 0 && (g.nx * sizeof(T)) % 32 == 0) ? 1u : 0u;
+        const unsigned grid = static_cast<unsigned>(g.T ? g.T : 1);
         decompress_nd_tile_kernel<T, NDIM><<<grid, NT, smem, st>>>(static_cast<const uint8_t *>(d_cmp),
-                                                                   static_cast<T *>(d_out), g0, d_status);
+                                                                   static_cast<T *>(d_out), g, d_status);
         return launch_status();
     } else {
         constexpr int smem = ND_DRING + 64;
         if (int rc = set_smem(decompress_nd_kernel<T, NDIM>, smem)) return rc;
         GeomND g = g0;
         nd_rows<T, NDIM>(g);
+        g.vec32 = (reinterpret_cast<uintptr_t>(d_out) % 32 == 0 && (g.nx * sizeof(T)) % 32 == 0) ? 1u : 0u;
         const unsigned grid = persistent_grid(decompress_nd_kernel<T, NDIM>, NT, smem, g.T);
         decompress_nd_kernel<T, NDIM><<<grid, NT, smem, st>>>(static_cast<const uint8_t *>(d_cmp),
                                                               static_cast<T *>(d_out), g, d_status);

@@ -45,7 +45,27 @@ struct GeomND {
     uint64_t roff[16];      // compression gathers: byte offset of block row r (r = iy + BY iz)
     uint64_t ystep, zstep;  // the same as steps: row r-1 -> r within / across a z-plane
     uint32_t vec;           // rows are whole 16-byte vectors (nx % (16/w) == 0)
+    uint32_t vec32;         // rows start 32-byte aligned (field base and nx * w): 256-bit accesses
 };
+
+// 32-byte (256-bit) global accesses, sm_100: LDG.E.ENL2.256 / STG.E.ENL2.256
+__device__ __forceinline__ void ld32B(const double *p, double (&v)[4]) {
+    asm volatile("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];" : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(p));
+}
+__device__ __forceinline__ void ld32B(const float *p, float (&v)[8]) {
+    asm volatile("ld.global.nc.v8.f32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+                 : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]), "=f"(v[4]), "=f"(v[5]), "=f"(v[6]), "=f"(v[7])
+                 : "l"(p));
+}
+__device__ __forceinline__ void st32B_cs(double *p, const double (&v)[4]) {
+    asm volatile("st.global.cs.v4.f64 [%0], {%1, %2, %3, %4};" ::"l"(p), "d"(v[0]), "d"(v[1]), "d"(v[2]), "d"(v[3])
+                 : "memory");
+}
+__device__ __forceinline__ void st32B_cs(float *p, const float (&v)[8]) {
+    asm volatile("st.global.cs.v8.f32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(p), "f"(v[0]), "f"(v[1]),
+                 "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7])
+                 : "memory");
+}
 
 template <int NDIM>
 struct BlockShape;
@@ -157,7 +177,24 @@ __device__ __forceinline__ void gather_block(const T *__restrict__ in, const Geo
     uint64_t outb = 0;
     if (g.vec) {
         const bool interior = active && x0 + S::BX <= g.nx && y0 + S::BY <= g.ny && z0 + S::BZ <= g.nz;
-        if (interior) {
+        constexpr bool ROW32 = (S::BX * sizeof(T)) % 32 == 0;  // rows of whole 32-byte vectors
+        if (interior && ROW32 && g.vec32) {
+            // 256-bit loads (3D f64: one per row; 2D: two per row of 8 values)
+            constexpr int V32 = 32 / sizeof(T);
+            const char *rp = base;
+#pragma unroll
+            for (int r = 0; r < NROW; r++) {
+                if (sizeof(T) == 8 && r && (r * S::BX) % 16 == 0) asm volatile("" ::: "memory");
+                if (r) rp += (r % S::BY) ? g.ystep : g.zstep;
+#pragma unroll
+                for (int u = 0; u < S::BX / V32; u++) {
+                    T tmp[V32];
+                    ld32B(reinterpret_cast<const T *>(rp) + u * V32, tmp);
+#pragma unroll
+                    for (int k = 0; k < V32; k++) v[r * S::BX + u * V32 + k] = qpattern<NDIM, CHECKED>(tmp[k], inv, bad);
+                }
+            }
+        } else if (interior) {
             // rows by a chain of pointer steps (so that the 16 row addresses are never
             // all live at once: 64 values + 32 address registers would spill)
             const char *rp = base;
@@ -868,8 +905,20 @@ __global__ void __launch_bounds__(NT, 2) decompress_nd_kernel(const uint8_t *__r
         char *base = reinterpret_cast<char *>(out) + ((static_cast<uint64_t>(z0) * g.ny + y0) * g.nx + x0) * sizeof(T);
         const bool interior = active && g.vec && x0 + S::BX <= g.nx && y0 + S::BY <= g.ny && z0 + S::BZ <= g.nz;
         char *rp = base;
+        constexpr bool ROW32 = (S::BX * sizeof(T)) % 32 == 0;  // 2D f32 rows: one 256-bit store
+        const bool wide = ROW32 && g.vec32;
         inv_lorenzo_block<NDIM>(v, [&](int r) {
-            if (interior) {
+            if (interior && wide) {
+                constexpr int V32 = 32 / sizeof(T);
+                if (r) rp += (r % S::BY) ? g.ystep : g.zstep;
+#pragma unroll
+                for (int u = 0; u < S::BX / V32; u++) {
+                    T tmp[V32];
+#pragma unroll
+                    for (int k = 0; k < V32; k++) tmp[k] = dequantize(static_cast<int>(v[r * S::BX + u * V32 + k]), K.s);
+                    st32B_cs(reinterpret_cast<T *>(rp) + u * V32, tmp);
+                }
+            } else if (interior) {
                 using VT = typename Vec16<T>::type;
                 constexpr int V = Vec16<T>::V;
                 if (r) rp += (r % S::BY) ? g.ystep : g.zstep;
@@ -1027,8 +1076,24 @@ __global__ void __launch_bounds__(NT, 3) decompress_nd_tile_kernel(const uint8_t
     }
     if (active) {
         const BlockOrigin bo = block_origin<NDIM>(g, b);
-        if (interior_vec<T, NDIM>(g, bo)) {
-            using S = BlockShape<NDIM>;
+        using S = BlockShape<NDIM>;
+        constexpr bool ROW32 = (S::BX * sizeof(T)) % 32 == 0;
+        if (ROW32 && g.vec32 && interior_vec<T, NDIM>(g, bo)) {
+            // 256-bit streaming stores (3D f64: one per row)
+            constexpr int V32 = 32 / sizeof(T);
+#pragma unroll
+            for (int r = 0; r < S::BY * S::BZ; r++) {
+                const int iy = r % S::BY, iz = r / S::BY;
+                T *row = out + ((bo.z0 + iz) * g.ny + bo.y0 + iy) * g.nx + bo.x0;
+#pragma unroll
+                for (int u = 0; u < S::BX / V32; u++) {
+                    T tmp[V32];
+#pragma unroll
+                    for (int k = 0; k < V32; k++) tmp[k] = dequantize(q[r * S::BX + u * V32 + k], K.s);
+                    st32B_cs(row + u * V32, tmp);
+                }
+            }
+        } else if (interior_vec<T, NDIM>(g, bo)) {
             using VT = typename Vec16<T>::type;
             constexpr int V = Vec16<T>::V;
 #pragma unroll

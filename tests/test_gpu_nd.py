@@ -249,3 +249,38 @@ def test_nd_lookback_window_width_same_stream(flags, dtype):
     np.testing.assert_array_equal(out[: ref.size].cpu().numpy(), ref)
     with pytest.raises(cz.CszpError):
         cz.compress_nd(x, 1e-4, "rel", "outlier", out=out, out_bytes=nb, flags=cz.FLAG_LB_WIDE | cz.FLAG_LB_NARROW)
+
+
+@pytest.mark.parametrize("shape,dtype", [((256, 1024), np.float32), ((96, 1000), np.float64),
+                                         ((24, 64, 128), np.float64), ((20, 40, 96), np.float64)])
+@pytest.mark.parametrize("offset16", [False, True])
+def test_nd_256bit_paths(shape, dtype, offset16):
+    """Rows of whole 32-byte vectors (2D: 8 values x w, 3D f64: 4 doubles) are gathered and
+    stored with 256-bit accesses when the field base and the row pitch are 32-byte aligned
+    (g.vec32); a base that is only 16-byte aligned takes the 16-byte path. Multi-tile
+    fields, both bases: streams and values equal the oracle's."""
+    xh = smooth_field(shape, sum(shape), dtype, noise=1e-2)
+    w = np.dtype(dtype).itemsize
+    pad = 16 // w if offset16 else 0
+    flat = torch.empty(xh.size + pad + 16, dtype=torch.float32 if w == 4 else torch.float64, device=DEV)
+    x = flat[pad: pad + xh.size].view(shape)
+    x.copy_(torch.from_numpy(xh))
+    assert (x.data_ptr() % 32 == 16) == offset16
+    ref, rc = oracle.compress_nd(xh, 1e-4, oracle.REL, oracle.OUTLIER)
+    assert rc == oracle.OK
+    out = torch.full((cz.compress_bound_nd(xh.shape, x.dtype),), 0xAA, dtype=torch.uint8, device=DEV)
+    nb = torch.zeros(1, dtype=torch.int64, device=DEV)
+    cz.compress_nd(x, 1e-4, "rel", "outlier", out=out, out_bytes=nb)
+    torch.cuda.synchronize()
+    assert int(nb.item()) == ref.size
+    np.testing.assert_array_equal(out[: ref.size].cpu().numpy(), ref)
+    yflat = torch.full_like(flat, float("nan"))
+    y = yflat[pad: pad + xh.size].view(shape)
+    st = torch.zeros(1, dtype=torch.int32, device=DEV)
+    cz.decompress_nd(out, shape, x.dtype, out=y, status=st)
+    torch.cuda.synchronize()
+    assert int(st.item()) == 0
+    yr, rc = oracle.decompress_nd(ref, shape, dtype)
+    iv = np.uint32 if w == 4 else np.uint64
+    np.testing.assert_array_equal(y.cpu().numpy().view(iv), yr.view(iv))
+    assert torch.isnan(yflat[:pad]).all() and torch.isnan(yflat[pad + xh.size:]).all()  # nothing outside
