@@ -129,7 +129,8 @@ int cszp2_compress_prepare_range(const void *d_in, uint64_t n, int dtype, double
  *  LOAD_VEC and LOAD_SCALAR are exclusive (ARG otherwise).
  *  CSZP2_FLAG_LB_WIDE / CSZP2_FLAG_LB_NARROW: force the lookback's first window
  *    to 256 / 32 predecessors (by default 32 below 2^16 tiles, 256 from 2^16 on; a speed
- *    choice that changes no stream byte). Exclusive (ARG otherwise).
+ *    choice that changes no stream byte). Exclusive (ARG otherwise). They apply to the
+ *    TMA-load product path; the LOAD_* ablations keep 256, CHAINED_SCAN has no window.
  *  CSZP2_FLAG_PREPARED (not an ablation): the caller guarantees that a
  *    cszp2_compress_prepare(_range) on this d_out precedes this call on the stream
  *    with no encode in between, so the tile index and ticket are still zero and
