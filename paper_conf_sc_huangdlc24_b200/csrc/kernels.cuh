@@ -452,6 +452,38 @@ __device__ __forceinline__ uint32_t tile_scan_1bar(uint32_t v, bool bad, uint32_
     return (warp ? before : 0u) + inc - v;
 }
 
+// tile_scan_1bar split around a barrier the caller already has: part 1 (warp scan, warp
+// total + bad flag to s_warp) before it, part 2 (warp totals -> exclusive prefix, tile
+// total, OR of bad) after it.
+__device__ __forceinline__ uint32_t scan_part1(uint32_t v, bool bad, uint32_t *s_warp) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    uint32_t inc = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
+    }
+    const bool wbad = __any_sync(0xffffffffu, bad);
+    if (lane == 31) s_warp[warp] = inc | (wbad ? 0x80000000u : 0u);
+    return inc;
+}
+__device__ __forceinline__ uint32_t scan_part2(uint32_t v, uint32_t inc, const uint32_t *s_warp, uint32_t *total,
+                                               bool *any_bad) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    constexpr int NW = NT / 32;
+    const uint32_t raw = lane < NW ? s_warp[lane] : 0u;
+    *any_bad = __any_sync(0xffffffffu, (raw >> 31) != 0u);
+    uint32_t wt = raw & 0x7FFFFFFFu;
+#pragma unroll
+    for (int o = 1; o < NW; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, wt, o);
+        if (lane >= o) wt += y;
+    }
+    const uint32_t before = __shfl_sync(0xffffffffu, wt, (warp + NW - 1) % NW);
+    *total = __shfl_sync(0xffffffffu, wt, NW - 1);
+    return (warp ? before : 0u) + inc - v;
+}
+
 // ❸ Decoupled lookback (Fig 13; after Merrill & Garland [25]), split
 // so that no CTA ever sits on an unpublished tile while it waits:
 //   publish_aggregate: tile t announces (A | aggregate) — (P | aggregate) for

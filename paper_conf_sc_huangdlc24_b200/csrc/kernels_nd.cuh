@@ -666,7 +666,7 @@ __global__ void __launch_bounds__(NT, 2) decompress_nd_kernel(const uint8_t *__r
     extern __shared__ uint8_t stage_raw[];
     uint8_t *ring = smem_align<16>(stage_raw);
     __shared__ uint64_t s_bar[2];
-    __shared__ uint32_t s_warp[NT / 32];
+    __shared__ uint32_t s_warp[2][NT / 32];  // the scan's warp totals, by tile parity
     __shared__ uint64_t s_excl[2];
     __shared__ uint32_t s_bytes[2];
     __shared__ uint32_t s_rpos[2];
@@ -754,6 +754,25 @@ __global__ void __launch_bounds__(NT, 2) decompress_nd_kernel(const uint8_t *__r
         const uint64_t bn = (t + G) * BPT + tid;
         if (t + G < g.T && bn < g.nb) ob_next = cmp[g.O + bn];
     }
+    // block payload size and reserved-bit check from an offset byte (FORMAT.md §4)
+    auto bsize = [](uint32_t ob, bool &bad) {
+        const uint32_t f = ob & 31u;
+        const bool o = (ob & 0x80u) != 0;
+        bad = !o && (ob & 0x60u);
+        return o ? 8u + (((ob >> 5) & 3u) + 1u) + 8u * f : (f ? 8u * (1u + f) : 0u);
+    };
+    // The scan of a tile's 256 block sizes is computed one tile ahead (its offset bytes
+    // are prefetched), its warp totals crossing the CTA barrier that the current tile
+    // needs anyway: one barrier per tile instead of two.
+    uint32_t my_excl, agg;
+    bool any_bad;
+    {
+        bool bd;
+        const uint32_t sz = bsize(ob_cur, bd);
+        const uint32_t inc = scan_part1(sz, bd, s_warp[0]);
+        __syncthreads();
+        my_excl = scan_part2(sz, inc, s_warp[0], &agg, &any_bad);
+    }
     int err = 0;
     for (uint32_t it = 0; t < g.T; ++it, t += G) {
         const int cur = it & 1;
@@ -788,19 +807,16 @@ __global__ void __launch_bounds__(NT, 2) decompress_nd_kernel(const uint8_t *__r
         const uint32_t nob = is_o ? ((obyte >> 5) & 3u) + 1u : 0u;
         const bool bad = (!is_o && (obyte & 0x60u));
         const uint32_t size = is_o ? 8u + nob + 8u * fl : (fl ? 8u * (1u + fl) : 0u);
-        // one-barrier scan: s_warp is next rewritten after the CTA barrier below
-        uint32_t agg;
-        bool any_bad;
-        const uint32_t my_excl = tile_scan_1bar(size, bad, s_warp, &agg, &any_bad, 0);
+        (void)bad;
+        // the payload's arrival also orders thread 0's s_bytes / s_excl / s_rpos writes for
+        // this tile (its expect_tx arrival releases them), even when they were made after
+        // the last barrier (a deferred launch)
+        mbar_wait(&s_bar[cur], (it >> 1) & 1);
         if (any_bad || agg != s_bytes[cur]) {
             err = ST_FORMAT;
-            if (tid == 0) {
-                mbar_wait(&s_bar[cur], (it >> 1) & 1);
-                if (pending) mbar_wait(&s_bar[cur ^ 1], ((it + 1) >> 1) & 1);
-            }
+            if (tid == 0 && pending) mbar_wait(&s_bar[cur ^ 1], ((it + 1) >> 1) & 1);
             break;
         }
-        mbar_wait(&s_bar[cur], (it >> 1) & 1);
 
         // ---- ❷⁻¹: sign (8 B), outlier, planes (8 B each) -> residual magnitudes
         uint32_t v[LND];
@@ -871,11 +887,18 @@ __global__ void __launch_bounds__(NT, 2) decompress_nd_kernel(const uint8_t *__r
                 unpack_planes<5>(hi);
             }
         }
+        // the next tile's scan, part 1 (its warp totals cross the barrier below)
+        bool bad_n;
+        const uint32_t size_n = tn < g.T ? bsize(ob_next, bad_n) : (bad_n = false, 0u);
+        const uint32_t inc_n = scan_part1(size_n, bad_n, s_warp[cur ^ 1]);
         __syncthreads();  // every thread has read this tile's payload from the ring
         if (tid == 0 && deferred) {  // the ring is empty now: fetch the next payload
             launch(nraw_p, nraw_i, cur ^ 1, true);
             pending = true;
         }
+        uint32_t agg_n;
+        bool any_bad_n;
+        const uint32_t my_excl_n = scan_part2(size_n, inc_n, s_warp[cur ^ 1], &agg_n, &any_bad_n);
         if (is_o) lo[0] = outl;
 #pragma unroll
         for (int i = 0; i < 32; i++) {
@@ -940,6 +963,9 @@ __global__ void __launch_bounds__(NT, 2) decompress_nd_kernel(const uint8_t *__r
         });
         ob_cur = ob_next;
         ob_next = ob_pref;
+        my_excl = my_excl_n;
+        agg = agg_n;
+        any_bad = any_bad_n;
     }
     if (tid == 0 && err && d_status) atomicOr(d_status, err);
 }
